@@ -1,0 +1,114 @@
+"""Pins for the seeded generators and the graph recipe."""
+import os
+
+import numpy as np
+import pytest
+
+from workloads import prng
+from workloads.configs import TINY, GPT2S
+from workloads.inputs import molecule_slow, molecules, molecule_of, prompt_tokens, shuffle
+from oracle.numerics import is_bf16_exact
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _golden_ints(name):
+    with open(os.path.join(GOLDEN, name)) as f:
+        return [int(l) for l in f if l.strip() and not l.startswith("#")]
+
+
+def test_splitmix64_published_vector():
+    want = _golden_ints("splitmix64_1234567.txt")
+    assert [prng.draw_int(1234567, i) for i in range(5)] == want
+    got = prng.draw(np.uint64(1234567), np.arange(5, dtype=np.uint64))
+    assert [int(v) for v in got] == want
+
+
+def test_key_definition_composes_draws():
+    # key(s, st) = draw(s ^ draw(st, 0), 0): check against the scalar splitmix sequence
+    s, st = 0x7111, 37
+    inner = prng.splitmix64_sequence(st, 1)[0]
+    assert prng.key(s, st) == prng.splitmix64_sequence(s ^ inner, 1)[0]
+
+
+def test_weight_values_bf16_exact_and_uniform_levels():
+    w = prng.weight_values(0x6732, 5, 1 << 18)
+    assert is_bf16_exact(w)
+    lv = np.round(w * 4096).astype(np.int64)
+    assert np.array_equal(lv.astype(np.float32) / 4096, w)
+    assert lv.min() >= -128 and lv.max() <= 127
+    hist = np.bincount(lv + 128, minlength=256)
+    exp = len(w) / 256
+    chi2 = float(((hist - exp) ** 2 / exp).sum())
+    assert chi2 < 400, chi2       # 255 dof: mean 255, sd ~22.6
+
+
+def test_gain_values_range_bf16_exact():
+    g = prng.gain_values(0x7111, 23, 4096)
+    assert is_bf16_exact(g)
+    lv = np.round((g - 1) * 64).astype(np.int64)
+    assert lv.min() == -8 and lv.max() == 7
+    assert np.all(np.bincount(lv + 8, minlength=16) > 150)
+
+
+def test_prompt_tokens_in_range_and_seeded():
+    p = prompt_tokens(3, 2, 16, GPT2S.vocab)
+    assert p.shape == (2, 16) and p.dtype == np.int32
+    assert p.min() >= 0 and p.max() < GPT2S.vocab
+    assert not np.array_equal(p[0], p[1])
+    assert np.array_equal(p, prompt_tokens(3, 2, 16, GPT2S.vocab))
+    # definition: draw(key(seed, k*256+b), j) mod V
+    assert p[1, 5] == prng.draw_int(prng.key(0xC0FFEE, 3 * 256 + 1), 5) % GPT2S.vocab
+
+
+def _connected(n, edges):
+    adj = {i: set() for i in range(n)}
+    for u, v, _ in edges:
+        adj[u].add(v)
+        adj[v].add(u)
+    seen, stack = {0}, [0]
+    while stack:
+        x = stack.pop()
+        for y in adj[x]:
+            if y not in seen:
+                seen.add(y)
+                stack.append(y)
+    return len(seen) == n
+
+
+def test_molecule_generator_invariants_and_vectorised_equals_slow():
+    task = molecules(7, 64)
+    assert task["atom_off"][-1] == len(task["atom_type"])
+    assert task["edge_off"][-1] == len(task["edges"])
+    for m in range(64):
+        types, edges = molecule_of(task, m)
+        st, se = molecule_slow(7, m)
+        assert types == st and edges == se
+        n = len(types)
+        assert 10 <= n <= 30
+        assert all(0 <= t < 8 for t in types)
+        pairs = [(min(u, v), max(u, v)) for u, v, _ in edges]
+        assert all(u != v for u, v, _ in edges)
+        assert len(set(pairs)) == len(pairs)
+        assert all(0 <= b < 4 for _, _, b in edges)
+        assert n - 1 <= len(edges) <= n + 1
+        assert _connected(n, edges)
+
+
+def test_molecule_golden_first():
+    # frozen first molecule of task 1 (seed 0x6A5); regenerate only with a cited recipe change
+    types, edges = molecule_slow(1, 0)
+    with open(os.path.join(GOLDEN, "molecule_task1_mol0.txt")) as f:
+        lines = [l.strip() for l in f if l.strip() and not l.startswith("#")]
+    assert lines[0] == " ".join(map(str, types))
+    assert lines[1] == " ".join(f"{u},{v},{b}" for u, v, b in edges)
+
+
+def test_shuffle_is_permutation_and_fisher_yates_definition():
+    items = list(range(50))
+    out = shuffle(items)
+    assert sorted(out) == items and out != items
+    # two elements: i = 1, j = draw(key(42,0), 0) mod 2; items 1 and j swap (j = 0 swaps)
+    k = prng.key(42, 0)
+    want = ["b", "a"] if prng.draw_int(k, 0) % 2 == 0 else ["a", "b"]
+    assert shuffle(["a", "b"]) == want
