@@ -1,0 +1,365 @@
+#!/usr/bin/env python3
+"""Headline benchmark: multiplexed small-function throughput on B200 partitions.
+
+BASELINE.json metric: "tasks/sec and p50/p99 completion time vs #partitions;
+decode tok/s; HBM % peak". Workload = configs[1]: GPT-2-
+small-shaped Llama decode (random bf16 weights generated on device), batch 1,
+P = 16 prompt + G = 32 greedy tokens per task, 700 tasks per closed batch
+(§5.2: a fixed set of completions divided over the processes).
+
+One bench step = one closed batch of N_TASKS tasks submitted through the C ABI
+(fn_submit with host prompt buffers) and collected with fn_wait (host token
+buffers) on the chosen partition layout of each GPU. Before the timed run a
+short sweep measures the 1 / 2 / 4 / 7 / 14-partition layouts (D0 "fill").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--layout auto|1|2|4|7|14]
+    python bench.py --impl reference      # the CPU oracle on a bounded sample
+
+Multi-GPU (torchrun, one rank per GPU): tasks are independent, so every rank
+runs the same per-GPU batch on its own GPU (weak scaling, no data-path
+collective); rank 0 reports the total over ranks / the max span over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # before any CUDA init
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from workloads.configs import GPT2S, LAYOUTS_FILL, LAYOUTS_EQUAL  # noqa: E402
+from workloads.inputs import prompt_tokens  # noqa: E402
+
+P_LEN, G_LEN, N_TASKS = 16, 32, 700
+QUOTA = 512 << 20
+METRIC = "tasks/sec (p50/p99 completion, decode tok/s, HBM % peak) vs #partitions"
+UNIT = "tasks/s"
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def task_bytes(cfg, B, P, G):
+    """Algorithmic HBM bytes of one task (mirrors include/mx.h cost rule)."""
+    d, q, kv, ff = cfg.d_model, cfg.q_dim, cfg.kv_dim, cfg.d_ff
+    layer = 2 * (d * q + 2 * d * kv + q * d + 3 * d * ff) + 4 * d
+    head = 2 * cfg.vocab * d + 2 * d
+    S = P + G - 1
+    kvpos = cfg.n_layers * 2 * kv * 2
+    return (S * cfg.n_layers * layer + G * head + S * B * 2 * d + B * kvpos * (S * (S + 1) // 2)
+            + S * B * kvpos)
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_gpu{gpu}.csv")
+
+    def __enter__(self):
+        os.makedirs(os.path.dirname(self.path), exist_ok=True)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            self.proc.wait()
+            self.f.close()
+
+    def summary(self):
+        if not self.proc:
+            return None
+        sm, mx_, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        try:
+            for line in open(self.path):
+                c = [x.strip() for x in line.split(",")]
+                if len(c) < 9:
+                    continue
+                sm.append(float(c[1]))
+                mx_ = float(c[2])
+                for n, v in zip(names, c[5:9]):
+                    if v.lower().startswith("active"):
+                        reasons.add(n)
+        except Exception:
+            return None
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx_, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+# GPU arm
+# ---------------------------------------------------------------------------
+
+def make_layout(mx, gpu, n, kind):
+    sizes = (LAYOUTS_FILL if kind == "fill" else LAYOUTS_EQUAL)[n]
+    parts = [mx.part_create(gpu, s, QUOTA) for s in sizes]
+    return parts
+
+
+def run_batch(mx, fn, parts, n_tasks, equal_sizes, prompts):
+    """Submit a closed batch (all at t0) and wait for all. Returns per-task results."""
+    tasks = []
+    for k in range(1, n_tasks + 1):
+        t = mx.decode_task(fn, prompts[k - 1], G_LEN)
+        part = parts[(k - 1) % len(parts)] if equal_sizes else mx.MX_PART_ANY
+        mx.fn_submit(part, t)
+        tasks.append(t)
+    res = [mx.fn_wait(t) for t in tasks]
+    for r in res:
+        if r["status"] != 0:
+            raise RuntimeError(f"task {r['task']} failed with status {r['status']}")
+    return res, tasks
+
+
+def summarize(res, n_steps):
+    t_sub0 = min(r["t_submit_ns"] for r in res)
+    t_start = min(r["t_start_ns"] for r in res)
+    t_end = max(r["t_end_ns"] for r in res)
+    comp = [(r["t_end_ns"] - r["t_submit_ns"]) / 1e6 for r in res]
+    serv = [(r["t_end_ns"] - r["t_start_ns"]) / 1e6 for r in res]
+    return dict(span_s=(t_end - t_start) / 1e9, wall_s=(t_end - t_sub0) / 1e9,
+                p50_ms=float(np.percentile(comp, 50)), p99_ms=float(np.percentile(comp, 99)),
+                service_p50_ms=float(np.percentile(serv, 50)),
+                service_p99_ms=float(np.percentile(serv, 99)),
+                kernel_ms_mean=float(np.mean([r["kernel_ns"] for r in res]) / 1e6))
+
+
+def gpu_arm(args, rank, world, local_rank, dist):
+    from paper_conf_sc_dhakalrwercfm23_b200 import mx
+    mx.mx_init([local_rank])
+    gpu = 0
+    cfg = GPT2S
+    fn = mx.fn_register(mx.decode_desc(cfg))
+    prompts = [prompt_tokens(k, 1, P_LEN, cfg.vocab) for k in range(1, N_TASKS + 1)]
+    bytes_task = task_bytes(cfg, 1, P_LEN, G_LEN)
+    peak, peak_src = peaks()
+
+    def load(parts):
+        for p in parts:
+            mx.fn_load(fn, p)
+
+    # --- partition sweep (Fig. 4 analog: 1 vs 2/4/7/14 partitions) ----------------
+    sweep = []
+    sweep_tasks = 140
+    for n in (args.sweep if args.sweep else []):
+        parts = make_layout(mx, gpu, n, "fill")
+        load(parts)
+        eq = len(set(LAYOUTS_FILL[n])) == 1
+        run_batch(mx, fn, parts, min(sweep_tasks, 2 * len(parts)), eq, prompts)   # warm
+        res, _ = run_batch(mx, fn, parts, sweep_tasks, eq, prompts)
+        s = summarize(res, 1)
+        sweep.append(dict(partitions=n, sms=LAYOUTS_FILL[n], tasks=sweep_tasks,
+                          tasks_per_s=sweep_tasks / s["span_s"], p50_ms=s["p50_ms"],
+                          p99_ms=s["p99_ms"],
+                          hbm_frac=sweep_tasks * bytes_task / s["span_s"] / (peak * 1e9)))
+        for p in parts:
+            mx.part_destroy(p)
+    if args.layout == "auto":
+        n_main = max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 14
+    else:
+        n_main = int(args.layout)
+
+    # --- main timed run ------------------------------------------------------------
+    parts = make_layout(mx, gpu, n_main, "fill")
+    load(parts)
+    eq = len(set(LAYOUTS_FILL[n_main])) == 1
+    for _ in range(args.warmup):
+        run_batch(mx, fn, parts, N_TASKS, eq, prompts)
+    if dist:
+        dist.barrier()
+    l0 = mx.launch_count()
+    all_res = []
+    with ClockSampler(local_rank) as clk:
+        h0 = time.perf_counter()
+        for _ in range(args.steps):
+            res, _ = run_batch(mx, fn, parts, N_TASKS, eq, prompts)
+            all_res += res
+        h1 = time.perf_counter()
+    launches = mx.launch_count() - l0
+    if dist:
+        dist.barrier()
+    s = summarize(all_res, args.steps)
+    span = s["span_s"]
+    wall = h1 - h0
+    if dist:
+        import torch
+        t = torch.tensor([span, wall], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        span, wall = float(t[0]), float(t[1])
+    for p in parts:
+        mx.part_destroy(p)
+    mx.mx_shutdown()
+    if rank != 0:
+        return None
+    n_total = N_TASKS * args.steps * world
+    value = n_total / span
+    agg_bytes = bytes_task * N_TASKS * args.steps * world
+    achieved_gbs = agg_bytes / span / 1e9 / world   # per GPU
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "decode_traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    out = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(span / args.steps * 1e3, 3), "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "bf16 weights/KV, fp32 math",
+        "data": "synthetic (seeded bf16 weights generated on device, seeded prompts)",
+        "config": {"workload": "configs[1]: GPT-2-small-shaped Llama decode, batch 1, P=16, G=32",
+                   "model": "gpt2s-llama (L12 d768 H12 d_ff2048 V50257)",
+                   "tasks_per_step_per_gpu": N_TASKS, "partitions": n_main,
+                   "partition_sms": LAYOUTS_FILL[n_main],
+                   "placement": "STATIC (k-1) mod P" if eq else "WLAW (C5)",
+                   "parallelism": f"replicas x{world} (independent tasks, no collective)",
+                   "l2": "inputs larger than L2: 324 MB of weights per partition copy"},
+        "p50_ms": round(s["p50_ms"], 3), "p99_ms": round(s["p99_ms"], 3),
+        "service_p50_ms": round(s["service_p50_ms"], 3),
+        "service_p99_ms": round(s["service_p99_ms"], 3),
+        "gen_tok_per_s": round(value * G_LEN, 1),
+        "hbm_frac": round(achieved_gbs / peak, 4),
+        "partitions_sweep": sweep,
+        "roofline": {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak,
+                     "unit": "GB/s", "frac": round(achieved_gbs / peak, 4), "traffic": traffic,
+                     "kernel": "decode_kernel (persistent megakernel, all partitions together)",
+                     "algorithmic_bytes_per_launch": bytes_task,
+                     "kernel_ms_mean_per_launch": round(s["kernel_ms_mean"], 3),
+                     "peak_source": peak_src},
+        "e2e": {"value": round(n_total / wall, 3), "unit": UNIT,
+                "h2d_bytes_per_step": N_TASKS * world * P_LEN * 4,
+                "d2h_bytes_per_step": N_TASKS * world * (G_LEN * 4 + 24)},
+        "gpu_launches": int(launches) * world,
+        "timing": "value: device %globaltimer span (first kernel start -> last kernel end) "
+                  "over the K steps, max over ranks; kernel_ms from CUDA events on each "
+                  "partition's stream; e2e: host wall clock fn_submit -> last fn_wait",
+    }
+    if sweep:
+        base = [d for d in sweep if d["partitions"] == 1]
+        if base:
+            out["ratio_vs_1_partition"] = round(max(d["tasks_per_s"] for d in sweep)
+                                                / base[0]["tasks_per_s"], 3)
+    out["clocks"] = clk.summary()
+    if args.cpu_baseline and world == 1:
+        out["cpu_baseline"] = cpu_baseline(args)
+    return out
+
+
+# ---------------------------------------------------------------------------
+# CPU oracle (cpu_baseline leg and --impl reference arm)
+# ---------------------------------------------------------------------------
+
+def _threads():
+    try:
+        from threadpoolctl import threadpool_info
+        info = threadpool_info()
+        return max([i.get("num_threads", 1) for i in info] or [1])
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def cpu_baseline(args, n_tasks: int = 1):
+    from oracle import decode as od
+    from workloads.weights import decode_weights
+    w = decode_weights(GPT2S)
+    t0 = time.perf_counter()
+    for k in range(1, n_tasks + 1):
+        od.greedy_task(GPT2S, w, prompt_tokens(k, 1, P_LEN, GPT2S.vocab), G_LEN)
+    dt = time.perf_counter() - t0
+    return {"value": round(n_tasks / dt, 5), "unit": UNIT, "cores": _threads(), "kind": "oracle",
+            "sample": f"{n_tasks} full task(s) of the same workload (GPT-2s decode, P=16, G=32), "
+                      f"fp64 NumPy oracle, weight generation excluded; {dt:.1f} s"}
+
+
+def reference_arm(args, rank, world):
+    if rank != 0:
+        return None
+    from oracle import decode as od
+    from workloads.weights import decode_weights
+    w = decode_weights(GPT2S)
+    for k in range(args.warmup):
+        od.greedy_task(GPT2S, w, prompt_tokens(k + 1, 1, P_LEN, GPT2S.vocab), G_LEN)
+    t0 = time.perf_counter()
+    for k in range(args.steps):
+        od.greedy_task(GPT2S, w, prompt_tokens(k + 1, 1, P_LEN, GPT2S.vocab), G_LEN)
+    dt = time.perf_counter() - t0
+    v = args.steps / dt
+    cores = _threads()
+    return {"impl": "reference", "metric": METRIC, "value": round(v, 5), "unit": UNIT,
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(dt / args.steps * 1e3, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": "configs[1]: GPT-2-small-shaped Llama decode, batch 1, P=16, G=32",
+                       "sample": "1 task per step on the host CPU"},
+            "cpu_baseline": {"value": round(v, 5), "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": "1 full task per step (fp64 NumPy oracle)"},
+            "e2e": {"value": round(v, 5), "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="mx", choices=["mx", "reference"])
+    ap.add_argument("--layout", default="auto")
+    ap.add_argument("--sweep", default="1,2,4,7,14",
+                    help="comma list of partition counts for the pre-run sweep ('' = none)")
+    ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
+    args = ap.parse_args()
+    args.sweep = [int(x) for x in args.sweep.split(",") if x.strip()]
+    if args.warmup < 3 and args.impl == "mx":
+        print("warning: the timing rules want >= 3 warm-up steps", file=sys.stderr)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    dist = None
+    if world > 1:
+        import torch.distributed as tdist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        tdist.init_process_group("gloo", rank=rank, world_size=world)
+        dist = tdist
+    if args.impl == "reference":
+        out = reference_arm(args, rank, world)
+    else:
+        out = gpu_arm(args, rank, world, local_rank, dist)
+    if out is not None:
+        print(json.dumps(out), flush=True)
+    if dist:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

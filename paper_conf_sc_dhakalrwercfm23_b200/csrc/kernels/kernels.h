@@ -1,0 +1,96 @@
+// Host-visible kernel parameter blocks and launch helpers (no CUDA types in
+// the signatures beyond the opaque stream handle).
+#pragma once
+
+#include <cstdint>
+
+namespace mxk {
+
+constexpr int kStageBytes = 32768;      // one TMA bulk stage of weight rows
+constexpr int kConsumerWarps = 12;      // GEMV / attention warps per CTA
+constexpr int kDecodeThreads = 32 * (kConsumerWarps + 1);  // + 1 producer (TMA) warp
+constexpr int kMaxUnits = 128;          // (row, 256-col chunk) work units per tile
+constexpr int kMaxCtas = 160;           // >= 148 SMs
+constexpr int kMaxSeqCap = 512;         // attention keeps <= 16 scores per lane
+constexpr int kXinBytesCap = 96 * 1024; // activation staging (B * K * 4)
+
+// One decode task on one partition: all P+G-1 steps in ONE persistent launch
+// (grid = the partition's SMs, one CTA per SM), phases separated by a
+// device-wide barrier on a per-slot counter.
+struct DecodeParams {
+  int L, d, H, Hkv, hd, ff, V, q_dim, kv_dim, qkv_rows, max_seq;
+  int B, P, G;
+  float eps;
+  int n_ctas;
+  // weights (bf16 bits)
+  const uint16_t* w_layers;  // layer 0 block
+  uint64_t layer_stride;     // elements between layer blocks
+  uint64_t off_wqkv, off_wo, off_wgate, off_wup, off_wdown, off_gattn, off_gmlp;
+  const uint16_t* g_final;
+  const uint16_t* lm_head;
+  const uint16_t* embed;
+  const float* rope_cs;      // [max_seq][hd/2][2] (cos, sin)
+  // per-slot activations (fp32) and state
+  float* x;                  // [B][d] residual stream
+  float* qkv;                // [B][qkv_rows]
+  float* o;                  // [B][q_dim]
+  float* a;                  // [B][ff]
+  unsigned long long* cand;  // [kMaxCtas][B] per-CTA argmax keys
+  uint16_t* kc;              // [L][B][Hkv][max_seq][hd] bf16
+  uint16_t* vc;
+  const int* prompt;         // [B][P]
+  int* tokens;               // [B][G]
+  float* logits;             // [G][B][V] or nullptr
+  unsigned long long* bar;   // grid barrier counter (monotone across launches)
+  unsigned long long bar_base;
+  unsigned long long* stamps;  // [2] globaltimer start / end
+  int* err;                  // 0 ok, 1 barrier timeout
+};
+
+// Number of grid barriers one decode launch performs (host bookkeeping of bar_base).
+inline uint64_t decode_barriers(int L, int P, int G) {
+  uint64_t S = (uint64_t)(P + G - 1);
+  return S * 5ull * (uint64_t)L + (uint64_t)G;
+}
+
+// Shared-memory bytes of the decode kernel for a given shape.
+int decode_smem_bytes(int B, int kmax, int* n_stages);
+
+int launch_decode(const DecodeParams& p, void* stream);
+int launch_fill_weights(uint16_t* dst, uint64_t n, uint64_t seed, uint32_t tid, int is_gain,
+                        int n_ctas, void* stream);
+int launch_rope_table(float* dst, int max_seq, int hd, float theta, void* stream);
+int launch_probe(uint32_t* smids, int n_ctas, uint64_t spin_ns, void* stream);
+
+// IP-emulator MPNN (C4): grid = partition SMs, molecules strided over CTAs.
+struct MpnnParams {
+  int F, T, n_types, n_bonds;
+  int n_mol;
+  const uint16_t* e_atom;    // [n_types][F]
+  const uint16_t* w_b;       // [4][F][F]
+  const uint16_t* u;         // [F][F]
+  const uint16_t* c;         // [F]
+  const uint16_t* w1;        // [F][F]
+  const uint16_t* c1;        // [F]
+  const uint16_t* w2;        // [F]
+  const uint16_t* c2;        // [1]
+  const int* atom_off;       // [n_mol+1]
+  const uint8_t* atom_type;  // [n_atoms]
+  const int* edge_off;       // [n_mol+1]
+  const uint32_t* edges;     // packed mx_bond (6 B each) as raw bytes
+  float* out;                // [n_mol]
+  unsigned long long* stamps;
+  int n_ctas;
+};
+int mpnn_smem_bytes();
+int launch_mpnn(const MpnnParams& p, void* stream);
+
+uint64_t launch_counter();
+
+}  // namespace mxk
+
+namespace mxk {
+int launch_clock(unsigned long long* out, void* stream);
+int decode_set_attrs(int device);
+int mpnn_set_attrs(int device);
+}  // namespace mxk

@@ -1,0 +1,146 @@
+// Host runtime internals: devices, partitions (green contexts + arenas),
+// function instances, task slots, tasks and the per-GPU dispatcher.
+#pragma once
+
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <deque>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include <cuda.h>
+
+#include "../../include/mx.h"
+#include "arena.h"
+#include "kernels/kernels.h"
+#include "placement.h"
+
+namespace mx {
+
+uint64_t now_ns();
+void set_error(const char* fmt, ...);
+
+struct Gpu;
+struct Partition;
+struct FnInst;
+
+// One execution context of a partition: a green context over its SM groups
+// and one non-blocking stream (all of the partition's work is FIFO on it).
+struct Exec {
+  CUgreenCtx gctx = nullptr;
+  CUcontext ctx = nullptr;
+  CUstream stream = nullptr;
+  int n_ctas = 0;          // SMs provisioned (persistent grid size)
+  uint32_t epoch = 0;
+  CUevent ev[2][3] = {};   // per in-flight lane: kernel start, kernel end, done
+  int inflight = 0;
+};
+
+struct Task {
+  uint64_t id = 0;
+  int fn = 0;
+  int kind = 0;
+  int gpu = 0, part = 0;
+  uint64_t seq = 0;
+  uint32_t epoch = 0;
+  uint64_t cost = 0;
+  // decode
+  int B = 0, P = 0, G = 0;
+  std::vector<int32_t> prompt;
+  int32_t* out_tokens = nullptr;
+  float* out_logits = nullptr;
+  // mpnn
+  int n_mol = 0, n_atoms = 0, n_edges = 0;
+  std::vector<int32_t> atom_off, edge_off;
+  std::vector<uint8_t> atom_type, edges;
+  float* out_ip = nullptr;
+  // execution
+  bool ready = false;
+  FnInst* inst = nullptr;
+  int slot = -1;
+  Exec* exec = nullptr;
+  int lane = 0;
+  // completion
+  mx_status status = MX_OK;
+  bool done = false;
+  bool collected = false;
+  uint64_t t_submit = 0, t_start = 0, t_end = 0, kernel_ns = 0;
+};
+
+// Device + pinned-host buffers of one task slot of a function instance.
+struct Slot {
+  bool busy = false;
+  // decode
+  CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
+              logits = 0;
+  // mpnn
+  CUdeviceptr atom_off = 0, atom_type = 0, edge_off = 0, edges = 0, out = 0;
+  // common
+  CUdeviceptr bar = 0, stamps = 0, err = 0;
+  uint64_t bar_count = 0;
+  bool need_reset = false;
+  // pinned host staging
+  void* h_in = nullptr;
+  size_t h_in_bytes = 0;
+  void* h_out = nullptr;
+  size_t h_out_bytes = 0;
+  uint64_t* h_stamps = nullptr;   // [2] + err word
+};
+
+struct Fn {
+  int id = 0;
+  mx_fn_desc desc{};
+};
+
+struct FnInst {
+  Fn* fn = nullptr;
+  Partition* part = nullptr;
+  CUdeviceptr weights = 0;
+  uint64_t weight_bytes = 0;
+  CUdeviceptr rope = 0;
+  // decode layout (elements)
+  uint64_t layer_stride = 0, off_wqkv = 0, off_wo = 0, off_wgate = 0, off_wup = 0, off_wdown = 0,
+           off_gattn = 0, off_gmlp = 0, off_gfinal = 0, off_lm = 0, off_embed = 0;
+  // mpnn layout (elements)
+  uint64_t m_off[11] = {};
+  Slot slots[2];
+  bool loaded = false;
+};
+
+struct Partition {
+  int id = 0;
+  int gpu = 0;
+  bool live = true;
+  Arena arena;
+  CUdeviceptr sys = 0;     // small scratch (probe output)
+  std::unique_ptr<Exec> cur;
+  std::vector<std::unique_ptr<Exec>> draining;
+  std::deque<Task*> fifo;       // placed, not yet launched (seq order)
+  std::deque<Task*> inflight;   // launched, in order
+  std::map<int, std::unique_ptr<FnInst>> insts;
+  std::mutex load_mu;
+  uint64_t launches = 0;
+};
+
+struct Gpu {
+  int idx = 0, ordinal = 0;
+  CUdevice dev = 0;
+  CUcontext primary = nullptr;
+  int sm_total = 0, n_groups = 0, group_size = 8, remainder = 0, cc_major = 0, cc_minor = 0;
+  uint64_t mem_bytes = 0;
+  CUdevResource whole{};
+  std::vector<CUdevResource> groups;
+  int64_t clock_offset = 0;     // host_ns = device_ns + offset
+  std::thread thr;
+  std::mutex mu;                // guards partitions' queues / exec state on this GPU
+  std::condition_variable cv;
+  bool stop = false;
+  std::vector<Partition*> parts;
+};
+
+}  // namespace mx

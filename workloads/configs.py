@@ -112,18 +112,21 @@ C2 = DecodeWorkload(GPT2S, n_tasks=700, batch=1, prompt_len=16, gen_len=32)
 C3 = DecodeWorkload(LLAMA7B, n_tasks=100, batch=1, prompt_len=16, gen_len=32)
 MPNN_MOLS_PER_TASK = 1024
 
-# D0 partition layouts on 148 SMs in 8-SM groups ("fill" primary, "equal" MIG-like)
+# D0 partition layouts on 148 SMs. The library splits a B200 into 37 groups of
+# 4 SMs (green-context split ignoring SM co-scheduling; reading R8),
+# so "fill" layouts (MPS-like, primary) use all 148 SMs and "equal" layouts
+# (MIG-like fixed slices, §5.2) use identical sizes.
 LAYOUTS_FILL = {
     1: [148],
-    2: [72, 72],
-    4: [40, 40, 32, 32],
-    7: [24, 24, 24, 24, 16, 16, 16],
-    14: [16, 16, 16, 16] + [8] * 10,
+    2: [76, 72],
+    4: [40, 36, 36, 36],
+    7: [24, 24, 20, 20, 20, 20, 20],
+    14: [12] * 9 + [8] * 5,
 }
 LAYOUTS_EQUAL = {
     1: [148],
     2: [72, 72],
-    4: [32] * 4,
-    7: [16] * 7,
+    4: [36] * 4,
+    7: [20] * 7,
     14: [8] * 14,
 }
