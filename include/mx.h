@@ -216,6 +216,10 @@ mx_status mx_probe_smids(int32_t part, int32_t n_ctas, uint64_t spin_ns, uint32_
  * collect every CTA's SM id: smids[i*n_ctas + c] for parts[i].              */
 mx_status mx_probe_smids_concurrent(const int32_t* parts, int32_t n_parts, int32_t n_ctas,
                                     uint64_t spin_ns, uint32_t* smids);
+/* Per-CTA cycle buckets of the last decode launch on `part` when the library
+ * was initialised with MX_DECODE_PROF=1: [cta][8] = total, grid barrier,
+ * input staging, TMA-ring wait, GEMV, attention, producer wait, 0.       */
+mx_status mx_decode_profile(int32_t part, uint64_t* out, int32_t n_words);
 /* Number of kernels this library launched since init (all GPUs).          */
 mx_status mx_launch_count(uint64_t* out);
 

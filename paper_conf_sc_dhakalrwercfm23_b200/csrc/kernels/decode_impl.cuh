@@ -1,0 +1,923 @@
+// Persistent greedy-decode megakernel (sm_100a) — one launch runs a whole
+// decode task (all P+G-1 steps, all layers) on one partition.
+//
+// Method: Llama-style block, §3.2
+// P:113-115 (LLaMa2), §3.4 P:159 (20-word completions), §5.2 P:195 (100
+// paragraph completions). Per step s (position t = s), per layer l:
+//   QKV : h = RMSNorm(x, g_attn[l]);  qkv = [Wq;Wk;Wv] h
+//   ATT : q,k <- RoPE(t) (rotate-half, A11); Kc[l][t] = bf16(k), Vc[l][t] = bf16(v)
+//         (the only activation rounding point, A16); o_h = softmax(q.K/sqrt(hd)) V
+//   O   : x += Wo o
+//   GU  : h = RMSNorm(x, g_mlp[l]);  a = silu(Wgate h) * (Wup h)
+//   DOWN: x += Wdown a
+// then (steps s >= P-1 only) LM: logits = Wlm RMSNorm(x, g_final); token = argmax.
+//
+// B200 design:
+//  * grid = the partition's SMs (one CTA per SM); phases are separated by a
+//    device-wide barrier on a monotone counter (no floating-point atomics).
+//    When the attention is small (B*H*hd <= 1024) every CTA computes all heads
+//    itself as the O phase's input, removing one barrier per layer.
+//  * weights (>98% of the bytes) are streamed by a producer warp with 1-D TMA
+//    bulk copies (cp.async.bulk) into a shared-memory ring of 32 KB stages
+//    guarded by mbarriers. The weight stream is static, so the producer runs
+//    ahead ACROSS phase barriers.
+//  * 12 decoupled consumer warps: a work unit is (output row, <= 1024-column
+//    group); each lane owns 8 consecutive columns of each 256-column chunk
+//    (one 16-byte smem load), the activations are staged in a lane-permuted
+//    layout so both 16-byte activation loads are bank-conflict free, and each
+//    unit ends in one fixed shuffle tree. A row split over several units sums
+//    its partials in a fixed order. Every output row is owned by exactly one
+//    CTA, so results do not depend on the partition size.
+//  * rows are split across CTAs with a per-phase rotation so the per-CTA byte
+//    totals of a step stay balanced.
+#include <cfloat>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "launch.cuh"
+
+namespace mxk {
+
+enum PhaseKind { PH_QKV = 0, PH_ATT = 1, PH_O = 2, PH_GU = 3, PH_DOWN = 4, PH_LM = 5 };
+
+constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
+constexpr int kAttHd = 128;                 // max head_dim
+constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
+
+struct Phase {
+  int kind, layer, R, K, KP, NC, NG, TR;
+  const uint16_t* w0;
+  const uint16_t* w1;
+};
+
+__host__ __device__ __forceinline__ int round256(int k) { return (k + 255) & ~255; }
+
+__device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int layer) {
+  Phase ph;
+  ph.kind = kind;
+  ph.layer = layer;
+  ph.w1 = nullptr;
+  ph.w0 = nullptr;
+  ph.R = 0;
+  ph.K = 0;
+  const uint16_t* lw = p.w_layers + (uint64_t)layer * p.layer_stride;
+  switch (kind) {
+    case PH_QKV: ph.R = p.qkv_rows; ph.K = p.d; ph.w0 = lw + p.off_wqkv; break;
+    case PH_O: ph.R = p.d; ph.K = p.q_dim; ph.w0 = lw + p.off_wo; break;
+    case PH_GU: ph.R = p.ff; ph.K = p.d; ph.w0 = lw + p.off_wgate; ph.w1 = lw + p.off_wup; break;
+    case PH_DOWN: ph.R = p.d; ph.K = p.ff; ph.w0 = lw + p.off_wdown; break;
+    case PH_LM: ph.R = p.V; ph.K = p.d; ph.w0 = p.lm_head; break;
+    default: break;
+  }
+  ph.KP = round256(ph.K);
+  ph.NC = ph.KP / 256;
+  ph.NG = (ph.NC + kCPG - 1) / kCPG;
+  const int mult = (kind == PH_GU) ? 2 : 1;
+  int tr = 1;
+  if (ph.K > 0) {
+    tr = kStageBytes / (mult * ph.K * 2);
+    const int tr2 = kMaxUnits / (mult * ph.NG);
+    tr = max(1, min(tr, tr2));
+  }
+  ph.TR = tr;
+  return ph;
+}
+
+// Rows [r0, r1) of a phase owned by this CTA; `rot` rotates the assignment so
+// remainders land on different CTAs in different phases.
+__device__ __forceinline__ void my_rows(int R, int C, int cta, int rot, int* r0, int* r1) {
+  const int c = (cta + rot) % C;
+  *r0 = (int)(((long long)R * c) / C);
+  *r1 = (int)(((long long)R * (c + 1)) / C);
+}
+
+__host__ __device__ __forceinline__ int phases_per_layer(int fuse_att) { return fuse_att ? 4 : 5; }
+
+__device__ __forceinline__ int phase_kind(int k, int L, int fuse_att) {
+  const int pl = phases_per_layer(fuse_att);
+  if (k == pl * L) return PH_LM;
+  const int r = k % pl;
+  if (fuse_att) return r == 0 ? PH_QKV : r == 1 ? PH_O : r == 2 ? PH_GU : PH_DOWN;
+  return r;   // QKV, ATT, O, GU, DOWN
+}
+
+// Lane-permuted activation layout: within each 256-column chunk, lane l's
+// columns 8l..8l+3 live at [4l, 4l+4) and 8l+4..8l+7 at [128+4l, 128+4l+4).
+__device__ __forceinline__ int xidx(int b, int kk, int KP) {
+  const int c = kk >> 8, w = kk & 255, l = w >> 3, e = w & 7;
+  return b * KP + (c << 8) + ((e >> 2) << 7) + (l << 2) + (e & 3);
+}
+
+struct Smem {
+  uint8_t* ring;
+  float* xin;     // [B][KP] lane-permuted phase input
+  float* red;     // [n_stages][kMaxUnits][B] partial sums of multi-unit outputs
+  int* cnt;       // [n_stages][kMaxUnits] per-output completion counters
+  float* att;     // [kConsumerWarps][3][kAttHd]
+  uint64_t* full;
+  uint64_t* empty;
+  unsigned long long* best;  // [8]
+  int* tok;                  // [8]
+  float* wsum;               // [kConsumerWarps][8]
+};
+
+__device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int B, int kmax) {
+  Smem s;
+  uint8_t* p = base;
+  s.ring = p;
+  p += (size_t)n_stages * kStageBytes;
+  s.xin = reinterpret_cast<float*>(p);
+  p += (size_t)B * round256(kmax) * 4;
+  s.red = reinterpret_cast<float*>(p);
+  p += (size_t)n_stages * kMaxUnits * B * 4;
+  s.cnt = reinterpret_cast<int*>(p);
+  p += (size_t)n_stages * kMaxUnits * 4;
+  s.att = reinterpret_cast<float*>(p);
+  p += (size_t)kConsumerWarps * 3 * kAttHd * 4;
+  s.full = reinterpret_cast<uint64_t*>(p);
+  p += (size_t)n_stages * 8;
+  s.empty = reinterpret_cast<uint64_t*>(p);
+  p += (size_t)n_stages * 8;
+  s.best = reinterpret_cast<unsigned long long*>(p);
+  p += 8 * 8;
+  s.tok = reinterpret_cast<int*>(p);
+  p += 8 * 4;
+  s.wsum = reinterpret_cast<float*>(p);
+  return s;
+}
+
+int decode_smem_bytes(int B, int kmax, int* n_stages) {
+  const int fixed = B * round256(kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 + 8 * 4 +
+                    kConsumerWarps * 8 * 4 + 128;
+  const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
+  const int cap = 227 * 1024;
+  int ns = (cap - fixed) / per_stage;
+  if (ns > 6) ns = 6;
+  if (n_stages) *n_stages = ns;
+  if (ns < 2) return -1;
+  return ns * per_stage + fixed;
+}
+
+int decode_fuse_attention(int B, int H, int hd) { return (B * H * hd <= 1024) ? 1 : 0; }
+
+uint64_t decode_barriers(int L, int P, int G, int fuse_att) {
+  const uint64_t S = (uint64_t)(P + G - 1);
+  return S * (uint64_t)phases_per_layer(fuse_att) * (uint64_t)L + (uint64_t)G;
+}
+
+// Device-wide barrier among all CTAs of the launch (consumer warps only; the
+// producer warp never waits on it). A 4 s timeout sets *err; afterwards every
+// barrier passes without waiting, so a failed launch still terminates.
+__device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned long long target,
+                                             int tid_c) {
+  named_bar_sync(1, kNCT);
+  if (tid_c == 0) {
+    // release: this CTA's phase outputs (ordered before by bar.sync) become visible
+    asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(p.bar) : "memory");
+    if (!ld_volatile_i32(p.err)) {
+      const uint64_t t0 = globaltimer();
+      uint32_t spins = 0;
+      while (ld_relaxed_u64(p.bar) < target) {
+        if ((++spins & 255u) == 0) {
+          if (ld_volatile_i32(p.err)) break;
+          if (globaltimer() - t0 > 4000000000ull) {
+            atomicExch(p.err, 1);
+            break;
+          }
+        }
+      }
+    }
+    // acquire: one acquire load of the final count synchronizes with every CTA's
+    // release RMW (and invalidates this SM's L1 once for the whole CTA)
+    (void)ld_acquire_u64(p.bar);
+  }
+  named_bar_sync(1, kNCT);
+}
+
+// ---------------------------------------------------------------------------
+// Producer: stream this CTA's weight rows of every phase of every step.
+// ---------------------------------------------------------------------------
+__device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stages) {
+  const int C = p.n_ctas, cta = blockIdx.x, L = p.L;
+  const int S = p.P + p.G - 1;
+  const int pl = phases_per_layer(p.fuse_att);
+  uint32_t stage = 0, phase_bit = 0;
+  long long wait_cyc = 0;
+  const uint64_t pol = policy_evict_first();
+  for (int s = 0; s < S; ++s) {
+    const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
+    for (int k = 0; k < nph; ++k) {
+      const int kind = phase_kind(k, L, p.fuse_att);
+      if (kind == PH_ATT) continue;
+      const Phase ph = make_phase(p, kind, k / pl);
+      int r0, r1;
+      my_rows(ph.R, C, cta, k, &r0, &r1);
+      for (int r = r0; r < r1; r += ph.TR) {
+        const int n = min(ph.TR, r1 - r);
+        // never abandons the stream: after a barrier timeout the consumers run
+        // through the remaining phases without waiting, so every slot is freed.
+        const long long tw = clock64();
+        while (!mbar_try_wait_sleep(&sm.empty[stage], phase_bit ^ 1u, 20000u)) {
+        }
+        wait_cyc += clock64() - tw;
+        const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
+        const uint32_t total = (kind == PH_GU) ? 2u * one : one;
+        uint8_t* dst = sm.ring + (size_t)stage * kStageBytes;
+        mbar_arrive_expect_tx(&sm.full[stage], total);
+        bulk_g2s_evict_first(dst, ph.w0 + (size_t)r * ph.K, one, &sm.full[stage], pol);
+        if (kind == PH_GU)
+          bulk_g2s_evict_first(dst + one, ph.w1 + (size_t)r * ph.K, one, &sm.full[stage], pol);
+        if (++stage == (uint32_t)n_stages) {
+          stage = 0;
+          phase_bit ^= 1u;
+        }
+      }
+    }
+  }
+  if (p.prof) p.prof[cta * 8 + 6] = (unsigned long long)wait_cyc;
+}
+
+// ---------------------------------------------------------------------------
+// Attention for one (sequence b, head h) item by one warp. Writes o_h either to
+// global o (separate ATT phase) or into the lane-permuted O-phase input in
+// shared memory (fused). `writer` selects the single writer of Kc/Vc[t].
+// ---------------------------------------------------------------------------
+template <int B>
+__device__ __forceinline__ void attend(const DecodeParams& p, const Smem& sm, int layer, int t, int b, int h,
+                       bool writer, bool to_smem, int warp, int lane) {
+  const int Hkv = p.Hkv, hd = p.hd, half = hd / 2;
+  const int kvh = h / (p.H / Hkv);
+  float* qs = sm.att + warp * 3 * kAttHd;
+  float* ks = qs + kAttHd;
+  float* vs = ks + kAttHd;
+  const float scale_div = sqrtf((float)hd);
+  const float* base = p.qkv + (size_t)b * p.qkv_rows;
+  const size_t cache_row0 = ((((size_t)layer * B + b) * Hkv + kvh) * p.max_seq) * hd;
+  uint16_t* kcache = p.kc + cache_row0;
+  uint16_t* vcache = p.vc + cache_row0;
+  for (int i = lane; i < half; i += 32) {
+    const float c = p.rope_cs[((size_t)t * half + i) * 2 + 0];
+    const float sn = p.rope_cs[((size_t)t * half + i) * 2 + 1];
+    const float q1 = base[h * hd + i], q2 = base[h * hd + i + half];
+    qs[i] = q1 * c - q2 * sn;
+    qs[i + half] = q2 * c + q1 * sn;
+    const float* kb = base + p.q_dim + kvh * hd;
+    const float k1 = kb[i], k2 = kb[i + half];
+    const uint16_t kb1 = f32_to_bf16_rne(k1 * c - k2 * sn);
+    const uint16_t kb2 = f32_to_bf16_rne(k2 * c + k1 * sn);
+    const float* vb = base + p.q_dim + p.kv_dim + kvh * hd;
+    const uint16_t vb1 = f32_to_bf16_rne(vb[i]);
+    const uint16_t vb2 = f32_to_bf16_rne(vb[i + half]);
+    ks[i] = bf16_bits_to_f32(kb1);
+    ks[i + half] = bf16_bits_to_f32(kb2);
+    vs[i] = bf16_bits_to_f32(vb1);
+    vs[i + half] = bf16_bits_to_f32(vb2);
+    if (writer) {
+      kcache[(size_t)t * hd + i] = kb1;
+      kcache[(size_t)t * hd + i + half] = kb2;
+      vcache[(size_t)t * hd + i] = vb1;
+      vcache[(size_t)t * hd + i + half] = vb2;
+    }
+  }
+  __syncwarp();
+  // scores: lane owns keys j = lane + 32 m
+  float sc[kMaxSeqCap / 32];
+  float mx = -FLT_MAX;
+#pragma unroll
+  for (int m = 0; m < kMaxSeqCap / 32; ++m) {
+    sc[m] = -FLT_MAX;
+    if (32 * m <= t) {
+      const int j = lane + 32 * m;
+      if (j <= t) {
+        float dot = 0.f;
+        if (j < t) {
+          const uint16_t* kr = kcache + (size_t)j * hd;
+          for (int e = 0; e < hd; e += 8) {
+            const uint4 kv = *reinterpret_cast<const uint4*>(kr + e);
+            float kf[8];
+            unpack8(kv, kf);
+#pragma unroll
+            for (int q = 0; q < 8; ++q) dot = fmaf(qs[e + q], kf[q], dot);
+          }
+        } else {
+          for (int e = 0; e < hd; ++e) dot = fmaf(qs[e], ks[e], dot);
+        }
+        sc[m] = dot / scale_div;
+        mx = fmaxf(mx, sc[m]);
+      }
+    }
+  }
+  mx = warp_max(mx);
+  float e[kMaxSeqCap / 32];
+  float lsum = 0.f;
+#pragma unroll
+  for (int m = 0; m < kMaxSeqCap / 32; ++m) {
+    const int j = lane + 32 * m;
+    e[m] = (32 * m <= t && j <= t) ? expf(sc[m] - mx) : 0.f;
+    lsum += e[m];
+  }
+  const float sum = warp_sum(lsum);
+  // output: lane owns dims [lane*dpl, lane*dpl + dpl), dpl = hd/32; the value
+  // rows of up to 16 keys are loaded together, then consumed in key order.
+  const int dpl = hd >> 5;
+  float acc[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int m = 0; 32 * m <= t; ++m) {
+    float em = 0.f;
+#pragma unroll
+    for (int mm = 0; mm < kMaxSeqCap / 32; ++mm)
+      if (mm == m) em = e[mm];
+    const int jcnt = min(32, t + 1 - 32 * m);
+    for (int jj0 = 0; jj0 < jcnt; jj0 += 8) {
+      uint2 vr[8];
+#pragma unroll
+      for (int jj = 0; jj < 8; ++jj) {
+        const int j = 32 * m + jj0 + jj;
+        vr[jj] = make_uint2(0u, 0u);
+        if (jj0 + jj < jcnt && j < t) {
+          const uint16_t* src = vcache + (size_t)j * hd + lane * dpl;
+          if (dpl == 4)
+            vr[jj] = *reinterpret_cast<const uint2*>(src);
+          else if (dpl == 2)
+            vr[jj].x = *reinterpret_cast<const uint32_t*>(src);
+          else
+            vr[jj].x = *src;
+        }
+      }
+#pragma unroll
+      for (int jj = 0; jj < 8; ++jj) {
+        const int j = 32 * m + jj0 + jj;
+        const float ej = __shfl_sync(0xffffffffu, em, (jj0 + jj) & 31);
+        if (jj0 + jj < jcnt) {
+          float v[4];
+          if (j == t) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) v[i] = (i < dpl) ? vs[lane * dpl + i] : 0.f;
+          } else {
+            v[0] = __uint_as_float(vr[jj].x << 16);
+            v[1] = __uint_as_float(vr[jj].x & 0xffff0000u);
+            v[2] = __uint_as_float(vr[jj].y << 16);
+            v[3] = __uint_as_float(vr[jj].y & 0xffff0000u);
+          }
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            if (i < dpl) acc[i] = fmaf(ej, v[i], acc[i]);
+        }
+      }
+    }
+  }
+  const int KP = round256(p.q_dim);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    if (i < dpl) {
+      const int dd = lane * dpl + i;
+      const float o = acc[i] / sum;
+      if (to_smem)
+        sm.xin[xidx(b, h * hd + dd, KP)] = o;
+      else
+        p.o[(size_t)b * p.q_dim + h * hd + dd] = o;
+    }
+  }
+  __syncwarp();
+}
+
+// Separate attention phase (large attention): items spread over all warps of all CTAs.
+template <int B>
+__device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer, int t,
+                                int tid_c) {
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int items = B * p.H;
+  const int stride = p.n_ctas * kConsumerWarps;
+  const int group = p.H / p.Hkv;
+  for (int it = blockIdx.x * kConsumerWarps + warp; it < items; it += stride) {
+    const int b = it / p.H, h = it - b * p.H;
+    attend<B>(p, sm, layer, t, b, h, (h % group) == 0, false, warp, lane);
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Phase input staging (RMSNorm'd where the block says so), lane-permuted.
+// ---------------------------------------------------------------------------
+template <int B>
+__device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& sm, int kind, int layer, int s,
+                            int K, int tid_c) {
+  const int cta = blockIdx.x, C = p.n_ctas;
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int KP = round256(K);
+  if (kind == PH_O && p.fuse_att) {
+    // every CTA computes all heads (small attention): o lands directly in xin
+    for (int b = 0; b < B; ++b)
+      for (int kk = K + tid_c; kk < KP; kk += kNCT) sm.xin[xidx(b, kk, KP)] = 0.f;
+    const int group = p.H / p.Hkv;
+    for (int it = warp; it < B * p.H; it += kConsumerWarps) {
+      const int b = it / p.H, h = it - b * p.H;
+      attend<B>(p, sm, layer, s, b, h, cta == 0 && (h % group) == 0, true, warp, lane);
+    }
+    named_bar_sync(1, kNCT);
+    return;
+  }
+  const uint16_t* gain = nullptr;
+  const uint16_t* emb = nullptr;   // layer-0 input: the embedding rows of the tokens
+  const float* src = nullptr;
+  if (kind == PH_QKV && layer == 0) {
+    // input token: prompt for s < P, else the argmax of step s-1 (reduced from
+    // the per-CTA candidates, identically in every CTA).
+    if (tid_c < B) {
+      int tok;
+      if (s < p.P) {
+        tok = p.prompt[tid_c * p.P + s];
+      } else {
+        unsigned long long best = 0;
+        for (int c = 0; c < C; ++c) {
+          const unsigned long long v = p.cand[c * B + tid_c];
+          best = v > best ? v : best;
+        }
+        tok = (int)argmax_key_index(best);
+        if (cta == 0) p.tokens[tid_c * p.G + (s - p.P)] = tok;
+      }
+      sm.tok[tid_c] = tok;
+    }
+    named_bar_sync(1, kNCT);
+    emb = p.embed;
+    gain = p.w_layers + p.off_gattn;
+  } else {
+    src = (kind == PH_O) ? p.o : (kind == PH_DOWN) ? p.a : p.x;
+    if (kind == PH_QKV) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gattn;
+    if (kind == PH_GU) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gmlp;
+    if (kind == PH_LM) gain = p.g_final;
+  }
+  // Inputs are read once into registers (up to kRegVals per thread), then the
+  // RMSNorm scale is applied on the way into the lane-permuted smem layout.
+  constexpr int kRegVals = 8;
+  const bool in_regs = (B == 1) && (KP <= kRegVals * kNCT);
+  float rv[kRegVals];
+  float inv[B];
+#pragma unroll
+  for (int b = 0; b < B; ++b) inv[b] = 1.f;
+  auto load_in = [&](int b, int kk) -> float {
+    return emb ? bf16_bits_to_f32(emb[(size_t)sm.tok[b] * K + kk]) : src[b * K + kk];
+  };
+  if (in_regs) {
+#pragma unroll
+    for (int i = 0; i < kRegVals; ++i) {
+      const int kk = tid_c + i * kNCT;
+      rv[i] = (kk < K) ? load_in(0, kk) : 0.f;
+    }
+  }
+  if (gain) {
+    // RMSNorm (normalise, then scale; eps inside the sqrt): fixed-order block sum.
+    float part[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) part[b] = 0.f;
+    if (in_regs) {
+#pragma unroll
+      for (int i = 0; i < kRegVals; ++i) {
+        part[0] = fmaf(rv[i], rv[i], part[0]);
+      }
+    } else {
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+        for (int kk = tid_c; kk < K; kk += kNCT) {
+          const float v = load_in(b, kk);
+          part[b] = fmaf(v, v, part[b]);
+        }
+    }
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      part[b] = warp_sum(part[b]);
+      if (lane == 0) sm.wsum[warp * 8 + b] = part[b];
+    }
+    named_bar_sync(1, kNCT);
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      float t = 0.f;
+      for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + b];
+      inv[b] = 1.0f / sqrtf(t / (float)K + p.eps);
+    }
+  }
+  if (in_regs) {
+#pragma unroll
+    for (int i = 0; i < kRegVals; ++i) {
+      const int kk = tid_c + i * kNCT;
+      if (kk < KP) {
+        float v = rv[i];
+        if (kk < K) {
+          if (emb && cta == 0) p.x[kk] = v;
+          if (gain) v = v * inv[0] * bf16_bits_to_f32(gain[kk]);
+        }
+        sm.xin[xidx(0, kk, KP)] = v;
+      }
+    }
+  } else {
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      for (int kk = tid_c; kk < KP; kk += kNCT) {
+        float v = 0.f;
+        if (kk < K) {
+          v = load_in(b, kk);
+          if (emb && cta == 0) p.x[b * p.d + kk] = v;
+          if (gain) v = v * inv[b] * bf16_bits_to_f32(gain[kk]);
+        }
+        sm.xin[xidx(b, kk, KP)] = v;
+      }
+    }
+  }
+  named_bar_sync(1, kNCT);
+}
+
+// ---------------------------------------------------------------------------
+// GEMV phase over this CTA's rows, consuming the TMA ring. Warps are decoupled:
+// each warp waits for a stage, processes its work units of that stage, and
+// releases the stage on its own (the empty barrier counts kConsumerWarps
+// arrivals); there is no CTA-wide barrier per tile.
+//
+// A work unit is NR rows (B<=2: 4, B<=4: 2, else 1; GU: NR/2 gate/up output
+// pairs) over one group of <= kCPG 256-column chunks. Each lane owns 8
+// consecutive columns per chunk (one 16-byte smem load per row), the
+// activation loads are shared by the unit's rows, and the unit ends in NR
+// interleaved shuffle trees. When a row spans several groups (K > kCPG*256),
+// the group partials go through shared memory and the warp completing the last
+// one sums them in group order — every output is computed in one fixed order.
+// ---------------------------------------------------------------------------
+template <int B>
+struct RowsPerUnit {
+  static constexpr int value = (B <= 2) ? 4 : (B <= 4 ? 2 : 1);
+};
+
+template <int B, int NR, int NCH>
+__device__ __forceinline__ void multi_dot(const uint16_t* const (&w)[NR], const bool (&has)[NR],
+                                          const float* __restrict__ xc, int KP, int col0, int K,
+                                          int lane, float (&out)[NR][B]) {
+  // acc.x sums the even columns of the lane's 8, acc.y the odd ones (FFMA2)
+  unsigned long long acc[NR][B];
+#pragma unroll
+  for (int r = 0; r < NR; ++r)
+#pragma unroll
+    for (int b = 0; b < B; ++b) acc[r][b] = 0ull;
+  constexpr int CB = (NR >= 4) ? 1 : (NR == 2 ? 2 : 4);   // chunks per load batch (bounds registers)
+#pragma unroll
+  for (int cb = 0; cb < NCH; cb += CB) {
+    uint4 wv[CB][NR];
+#pragma unroll
+    for (int i = 0; i < CB; ++i) {
+      const int c = cb + i;
+      if (c < NCH) {
+        const int col = col0 + c * 256 + lane * 8;
+        const bool ok = (c < NCH - 1) || col < K;   // only the last chunk can be ragged
+#pragma unroll
+        for (int r = 0; r < NR; ++r)
+          wv[i][r] = (ok && has[r]) ? *reinterpret_cast<const uint4*>(w[r] + col)
+                                    : make_uint4(0, 0, 0, 0);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < CB; ++i) {
+      const int c = cb + i;
+      if (c < NCH) {
+#pragma unroll
+        for (int b = 0; b < B; ++b) {
+          const float4 x0 = *reinterpret_cast<const float4*>(xc + c * 256 + b * KP);
+          const float4 x1 = *reinterpret_cast<const float4*>(xc + c * 256 + b * KP + 128);
+#pragma unroll
+          for (int r = 0; r < NR; ++r) {
+            float f[8];
+            unpack8(wv[i][r], f);
+            ffma2(acc[r][b], f[0], f[1], x0.x, x0.y);
+            ffma2(acc[r][b], f[2], f[3], x0.z, x0.w);
+            ffma2(acc[r][b], f[4], f[5], x1.x, x1.y);
+            ffma2(acc[r][b], f[6], f[7], x1.z, x1.w);
+          }
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int r = 0; r < NR; ++r)
+#pragma unroll
+    for (int b = 0; b < B; ++b) out[r][b] = f32x2_sum(acc[r][b]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+    for (int r = 0; r < NR; ++r)
+#pragma unroll
+      for (int b = 0; b < B; ++b) out[r][b] += __shfl_xor_sync(0xffffffffu, out[r][b], o);
+}
+
+template <int B, int NR>
+__device__ __forceinline__ void multi_dot_n(int nch, const uint16_t* const (&w)[NR],
+                                            const bool (&has)[NR], const float* xc, int KP,
+                                            int col0, int K, int lane, float (&out)[NR][B]) {
+  switch (nch) {
+    case 1: multi_dot<B, NR, 1>(w, has, xc, KP, col0, K, lane, out); break;
+    case 2: multi_dot<B, NR, 2>(w, has, xc, KP, col0, K, lane, out); break;
+    case 3: multi_dot<B, NR, 3>(w, has, xc, KP, col0, K, lane, out); break;
+    case 4: multi_dot<B, NR, 4>(w, has, xc, KP, col0, K, lane, out); break;
+    case 5: multi_dot<B, NR, 5>(w, has, xc, KP, col0, K, lane, out); break;
+    case 6: multi_dot<B, NR, 6>(w, has, xc, KP, col0, K, lane, out); break;
+    case 7: multi_dot<B, NR, 7>(w, has, xc, KP, col0, K, lane, out); break;
+    default: multi_dot<B, NR, 8>(w, has, xc, KP, col0, K, lane, out); break;
+  }
+}
+
+template <int B, int NR, int KIND>
+__device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                              int k, int s,
+                              int tid_c, uint32_t& stage, uint32_t& phase_bit, int n_stages,
+                              long long& wait_cyc) {
+  const int C = p.n_ctas, cta = blockIdx.x;
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int K = ph.K, KP = ph.KP, NC = ph.NC, NG = ph.NG;
+  constexpr bool gu = (KIND == PH_GU);
+  constexpr bool resid = (KIND == PH_O || KIND == PH_DOWN);
+  constexpr int OPU_GU = NR / 2;            // GU outputs per unit (gate + up rows)
+  int r0, r1;
+  my_rows(ph.R, C, cta, k, &r0, &r1);
+  if (KIND == PH_LM) {
+    if (tid_c < B) sm.best[tid_c] = 0ull;
+    named_bar_sync(1, kNCT);
+  }
+  int start = 0;   // first warp of the current tile (rotates the assignment across tiles)
+  for (int r = r0; r < r1; r += ph.TR) {
+    const int n = min(ph.TR, r1 - r);
+    const int per = gu ? OPU_GU : NR;        // outputs per unit
+    const int groups = (n + per - 1) / per;
+    const int units = groups * NG;
+    int u = warp - start;
+    if (u < 0) u += kConsumerWarps;
+    start = (start + units) % kConsumerWarps;
+    // every warp observes the stage fill before releasing it (keeps the empty
+    // barrier's arrival count per round exact)
+    const long long tw = clock64();
+    while (!mbar_try_wait_sleep(&sm.full[stage], phase_bit, 20000u)) {
+    }
+    wait_cyc += clock64() - tw;
+    const uint16_t* wt = reinterpret_cast<const uint16_t*>(sm.ring + (size_t)stage * kStageBytes);
+    float* red = sm.red + (size_t)stage * kMaxUnits * B;
+    int* cnt = sm.cnt + stage * kMaxUnits;
+    for (; u < units; u += kConsumerWarps) {
+      const int gi = (NG == 1) ? u : u / NG;   // output group within the tile
+      const int g = u - gi * NG;
+      const int j0 = gi * per;                 // first tile-local output of the unit
+      const uint16_t* w[NR];
+      bool has[NR];
+#pragma unroll
+      for (int q = 0; q < NR; ++q) {
+        if (gu) {
+          const int j = j0 + (q >> 1);
+          has[q] = j < n;
+          w[q] = wt + (size_t)((q & 1) ? n + j : j) * K;
+        } else {
+          const int j = j0 + q;
+          has[q] = j < n;
+          w[q] = wt + (size_t)j * K;
+        }
+      }
+      // residual rows prefetched before the dot product (latency hidden)
+      float res[NR];
+#pragma unroll
+      for (int q = 0; q < NR; ++q) res[q] = 0.f;
+      if (resid && NG == 1 && lane < B) {
+#pragma unroll
+        for (int q = 0; q < NR; ++q)
+          if (has[q]) res[q] = p.x[lane * p.d + r + j0 + q];
+      }
+      const int c0 = g * kCPG;
+      float out[NR][B];
+      multi_dot_n<B, NR>(min(kCPG, NC - c0), w, has, sm.xin + c0 * 256 + 4 * lane, KP, c0 * 256, K,
+                         lane, out);
+      if (NG > 1) {
+        // group partials -> smem; the last arriving warp finishes the unit's outputs
+        if (lane == 0) {
+#pragma unroll
+          for (int q = 0; q < NR; ++q)
+#pragma unroll
+            for (int b = 0; b < B; ++b) red[(u * NR + q) * B + b] = out[q][b];
+        }
+        __threadfence_block();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(&cnt[gi], 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old != NG - 1) continue;
+        __threadfence_block();
+#pragma unroll
+        for (int q = 0; q < NR; ++q)
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            float v = 0.f;
+            for (int gg = 0; gg < NG; ++gg) v += red[((gi * NG + gg) * NR + q) * B + b];
+            out[q][b] = v;
+          }
+        if (lane == 0) cnt[gi] = 0;   // reset for the stage's next round
+        if (resid && lane < B) {
+#pragma unroll
+          for (int q = 0; q < NR; ++q)
+            if (has[q]) res[q] = p.x[lane * p.d + r + j0 + q];
+        }
+      }
+      if (lane < B) {
+        const int b = lane;
+        float v[NR];
+#pragma unroll
+        for (int q = 0; q < NR; ++q) {
+          v[q] = out[q][0];
+#pragma unroll
+          for (int bb = 1; bb < B; ++bb)
+            if (bb == b) v[q] = out[q][bb];
+        }
+        switch (KIND) {
+          case PH_QKV:
+#pragma unroll
+            for (int q = 0; q < NR; ++q)
+              if (has[q]) p.qkv[b * p.qkv_rows + r + j0 + q] = v[q];
+            break;
+          case PH_O:
+          case PH_DOWN:
+#pragma unroll
+            for (int q = 0; q < NR; ++q)
+              if (has[q]) p.x[b * p.d + r + j0 + q] = res[q] + v[q];
+            break;
+          case PH_GU:
+#pragma unroll
+            for (int q = 0; q < NR; q += 2)
+              if (has[q]) {
+                const float gt = v[q], up = v[q + 1];
+                p.a[b * p.ff + r + j0 + q / 2] = gt / (1.0f + expf(-gt)) * up;
+              }
+            break;
+          case PH_LM: {
+            unsigned long long kb = 0ull;
+#pragma unroll
+            for (int q = 0; q < NR; ++q)
+              if (has[q]) {
+                const int row = r + j0 + q;
+                const unsigned long long kq = argmax_key(v[q], (uint32_t)row);
+                kb = kq > kb ? kq : kb;
+                if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = v[q];
+              }
+            atomicMax(&sm.best[b], kb);
+          } break;
+          default: break;
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.empty[stage]);
+    if (++stage == (uint32_t)n_stages) {
+      stage = 0;
+      phase_bit ^= 1u;
+    }
+  }
+  if (KIND == PH_LM) {
+    named_bar_sync(1, kNCT);
+    if (tid_c < B) p.cand[cta * B + tid_c] = sm.best[tid_c];
+  }
+}
+
+template <int B>
+__device__ __forceinline__ void gemv_phase(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                           int k, int s, int tid_c, uint32_t& stage,
+                                           uint32_t& phase_bit, int n_stages, long long& wait_cyc) {
+  constexpr int NR = RowsPerUnit<B>::value;
+  constexpr int NRG = NR < 2 ? 2 : NR;   // GU units always hold gate/up pairs
+  switch (ph.kind) {
+    case PH_QKV:
+      gemv_phase_nr<B, NR, PH_QKV>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      break;
+    case PH_O:
+      gemv_phase_nr<B, NR, PH_O>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      break;
+    case PH_GU:
+      gemv_phase_nr<B, NRG, PH_GU>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      break;
+    case PH_DOWN:
+      gemv_phase_nr<B, NR, PH_DOWN>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      break;
+    default:
+      gemv_phase_nr<B, NR, PH_LM>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      break;
+  }
+}
+
+template <int B>
+__global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams p, int n_stages,
+                                                                   int kmax) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const Smem sm = carve(smem_raw, n_stages, B, kmax);
+  const int warp_id = threadIdx.x >> 5;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < n_stages; ++i) {
+      mbar_init(&sm.full[i], 1);
+      mbar_init(&sm.empty[i], kConsumerWarps);
+    }
+    fence_mbar_init();
+    if (blockIdx.x == 0) p.stamps[0] = globaltimer();
+  }
+  for (int i = threadIdx.x; i < n_stages * kMaxUnits; i += blockDim.x) sm.cnt[i] = 0;
+  __syncthreads();
+
+  if (warp_id == 0) {
+    if ((threadIdx.x & 31) == 0) producer_loop(p, sm, n_stages);
+    return;
+  }
+
+  const int tid_c = threadIdx.x - 32;
+  const int L = p.L, S = p.P + p.G - 1;
+  const int pl = phases_per_layer(p.fuse_att);
+  uint32_t stage = 0, phase_bit = 0;
+  unsigned long long target = p.bar_base;
+  long long c_bar = 0, c_stage = 0, c_wait = 0, c_gemv = 0, c_att = 0;
+  const long long t_begin = clock64();
+  for (int s = 0; s < S; ++s) {
+    const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
+    for (int k = 0; k < nph; ++k) {
+      const int kind = phase_kind(k, L, p.fuse_att);
+      const int layer = k / pl;
+      long long t0 = clock64();
+      if (kind == PH_ATT) {
+        attention_phase<B>(p, sm, layer, s, tid_c);
+        const long long t1 = clock64();
+        c_att += t1 - t0;
+        t0 = t1;
+      } else {
+        const Phase ph = make_phase(p, kind, layer);
+        stage_input<B>(p, sm, kind, layer, s, ph.K, tid_c);
+        const long long t1 = clock64();
+        if (kind == PH_O && p.fuse_att)
+          c_att += t1 - t0;
+        else
+          c_stage += t1 - t0;
+        gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait);
+        const long long t2 = clock64();
+        c_gemv += t2 - t1;
+        t0 = t2;
+      }
+      target += (unsigned long long)p.n_ctas;
+      grid_barrier(p, target, tid_c);
+      c_bar += clock64() - t0;
+    }
+  }
+  if (p.prof && tid_c == 0) {
+    unsigned long long* pr = p.prof + blockIdx.x * 8;
+    pr[0] = (unsigned long long)(clock64() - t_begin);
+    pr[1] = (unsigned long long)c_bar;
+    pr[2] = (unsigned long long)c_stage;
+    pr[3] = (unsigned long long)c_wait;
+    pr[4] = (unsigned long long)c_gemv;
+    pr[5] = (unsigned long long)c_att;
+  }
+  // final token (argmax of the last step)
+  if (blockIdx.x == 0) {
+    if (tid_c < B) {
+      unsigned long long best = 0;
+      for (int c = 0; c < p.n_ctas; ++c) {
+        const unsigned long long v = p.cand[c * B + tid_c];
+        best = v > best ? v : best;
+      }
+      p.tokens[tid_c * p.G + (p.G - 1)] = (int)argmax_key_index(best);
+    }
+    named_bar_sync(1, kNCT);
+    if (tid_c == 0) p.stamps[1] = globaltimer();
+  }
+}
+
+template <int B>
+static int launch_b(const DecodeParams& p, void* stream) {
+  const int kmax = max(max(p.d, p.q_dim), p.ff);
+  int ns = 0;
+  const int smem = decode_smem_bytes(B, kmax, &ns);
+  if (smem < 0) return -3;
+  DecodeParams pc = p;
+  int ns_arg = ns, kmax_arg = kmax;
+  void* args[] = {&pc, &ns_arg, &kmax_arg};
+  return launch_kernel(decode_kernel<B>, dim3(p.n_ctas), dim3(kDecodeThreads), (unsigned)smem,
+                       stream, args);
+}
+
+int launch_decode(const DecodeParams& p, void* stream) {
+  switch (p.B) {
+    case 1: return launch_b<1>(p, stream);
+    case 2: return launch_b<2>(p, stream);
+    case 3: return launch_b<3>(p, stream);
+    case 4: return launch_b<4>(p, stream);
+    case 5: return launch_b<5>(p, stream);
+    case 6: return launch_b<6>(p, stream);
+    case 7: return launch_b<7>(p, stream);
+    case 8: return launch_b<8>(p, stream);
+    default: return -4;
+  }
+}
+
+int decode_set_attrs(int device) {
+  const int cap = 227 * 1024;
+  int rc = 0;
+  rc |= set_max_smem(decode_kernel<1>, cap, device);
+  rc |= set_max_smem(decode_kernel<2>, cap, device);
+  rc |= set_max_smem(decode_kernel<3>, cap, device);
+  rc |= set_max_smem(decode_kernel<4>, cap, device);
+  rc |= set_max_smem(decode_kernel<5>, cap, device);
+  rc |= set_max_smem(decode_kernel<6>, cap, device);
+  rc |= set_max_smem(decode_kernel<7>, cap, device);
+  rc |= set_max_smem(decode_kernel<8>, cap, device);
+  return rc;
+}
+
+}  // namespace mxk

@@ -22,6 +22,7 @@ struct DecodeParams {
   int B, P, G;
   float eps;
   int n_ctas;
+  int fuse_att;              // attention computed per CTA inside the O phase
   // weights (bf16 bits)
   const uint16_t* w_layers;  // layer 0 block
   uint64_t layer_stride;     // elements between layer blocks
@@ -45,13 +46,13 @@ struct DecodeParams {
   unsigned long long bar_base;
   unsigned long long* stamps;  // [2] globaltimer start / end
   int* err;                  // 0 ok, 1 barrier timeout
+  unsigned long long* prof;  // [n_ctas][8] cycle buckets (MX_DECODE_PROF=1) or nullptr
 };
 
+// 1 if every CTA computes the whole attention itself (B*H*hd <= 1024).
+int decode_fuse_attention(int B, int H, int hd);
 // Number of grid barriers one decode launch performs (host bookkeeping of bar_base).
-inline uint64_t decode_barriers(int L, int P, int G) {
-  uint64_t S = (uint64_t)(P + G - 1);
-  return S * 5ull * (uint64_t)L + (uint64_t)G;
-}
+uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 
 // Shared-memory bytes of the decode kernel for a given shape.
 int decode_smem_bytes(int B, int kmax, int* n_stages);

@@ -96,6 +96,7 @@ struct Lib {
 };
 
 static std::mutex g_init_mu;
+static bool g_decode_prof = false;
 static Lib* g_lib = nullptr;
 
 // ---------------------------------------------------------------------------
@@ -159,7 +160,7 @@ static int validate_fn(const mx_fn_desc& d) {
       return MX_EINVAL;
     }
     const int kmax = std::max(std::max(c.d_model, q), c.d_ff);
-    if ((int64_t)c.max_batch * kmax * 4 > mxk::kXinBytesCap ||
+    if ((int64_t)c.max_batch * ((kmax + 255) / 256 * 256) * 4 > mxk::kXinBytesCap ||
         mxk::decode_smem_bytes(c.max_batch, kmax, nullptr) < 0) {
       set_error("decode cfg: max_batch * max(d, q_dim, d_ff) * 4 > 96 KiB activation staging");
       return MX_EINVAL;
@@ -566,6 +567,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.G = t->G;
     k.eps = c.rms_eps;
     k.n_ctas = e->n_ctas;
+    k.fuse_att = mxk::decode_fuse_attention(k.B, k.H, k.hd);
     const uint16_t* wb = reinterpret_cast<const uint16_t*>(fi->weights);
     k.w_layers = wb;
     k.layer_stride = fi->layer_stride;
@@ -594,6 +596,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.bar_base = s.bar_count;
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
     k.err = reinterpret_cast<int*>(s.err);
+    k.prof = g_decode_prof ? reinterpret_cast<unsigned long long*>(p.sys + 65536) : nullptr;
     CU_TRY(drv().cuEventRecord(ev[0], st));
     int rc = mxk::launch_decode(k, st);
     if (rc) {
@@ -601,7 +604,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
       return MX_EDEVICE;
     }
     CU_TRY(drv().cuEventRecord(ev[1], st));
-    s.bar_count += mxk::decode_barriers(k.L, k.P, k.G) * (uint64_t)k.n_ctas;
+    s.bar_count += mxk::decode_barriers(k.L, k.P, k.G, k.fuse_att) * (uint64_t)k.n_ctas;
     const size_t tb = (size_t)t->B * t->G * 4;
     CU_TRY(drv().cuMemcpyDtoHAsync(s.h_out, s.tokens, tb, st));
     if (t->out_logits)
@@ -843,6 +846,7 @@ static int init_impl(const std::vector<int>& ordinals) {
   std::lock_guard<std::mutex> lk(g_init_mu);
   if (g_lib) return MX_OK;
   setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
+  g_decode_prof = getenv("MX_DECODE_PROF") && atoi(getenv("MX_DECODE_PROF")) == 1;
   const char* why = nullptr;
   if (!drv().load(&why)) {
     set_error("%s (no CUDA driver?)", why ? why : "driver load failed");
@@ -1026,7 +1030,7 @@ mx_status part_create(int32_t gpu, int32_t sm_count, uint64_t hbm_bytes, int32_t
     set_error("arena reservation failed");
     return rc;
   }
-  rc = p->arena.alloc(64 * 1024, 256, &p->sys);
+  rc = p->arena.alloc(128 * 1024, 256, &p->sys);
   if (rc) {
     destroy_exec(p->cur.get());
     p->arena.release();
@@ -1421,6 +1425,21 @@ mx_status mx_probe_smids_concurrent(const int32_t* parts, int32_t n_parts, int32
   MX_REQUIRE_INIT();
   if (!parts) return MX_EINVAL;
   return probe_many(L, parts, n_parts, n_ctas, spin_ns, smids);
+}
+
+mx_status mx_decode_profile(int32_t part, uint64_t* out, int32_t n_words) {
+  MX_REQUIRE_INIT();
+  if (!out || n_words < 0 || n_words > 8192) return MX_EINVAL;
+  Partition* p;
+  {
+    std::lock_guard<std::mutex> lk(L->mu);
+    if (!L->sched->is_live(part)) return MX_EINVAL;
+    p = L->parts[part].get();
+  }
+  CtxGuard cg(L->gpus[p->gpu]->primary);
+  CU_TRY(drv().cuStreamSynchronize(p->cur->stream));
+  CU_TRY(drv().cuMemcpyDtoH(out, p->sys + 65536, (size_t)n_words * 8));
+  return MX_OK;
 }
 
 mx_status mx_launch_count(uint64_t* out) {

@@ -99,6 +99,7 @@ _SIGS = {
     "mx_probe_smids_concurrent": (C.c_int32, [C.POINTER(C.c_int32), C.c_int32, C.c_int32,
                                               C.c_uint64, C.POINTER(C.c_uint32)]),
     "mx_launch_count": (C.c_int32, [C.POINTER(C.c_uint64)]),
+    "mx_decode_profile": (C.c_int32, [C.c_int32, C.POINTER(C.c_uint64), C.c_int32]),
     "mx_sched_new": (C.c_void_p, [C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_uint64]),
     "mx_sched_free": (None, [C.c_void_p]),
     "mx_sched_create": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64,
@@ -320,6 +321,13 @@ def probe_smids_concurrent(parts, n_ctas: int, spin_ns: int = 2_000_000) -> np.n
                                            out.ctypes.data_as(C.POINTER(C.c_uint32))),
            "mx_probe_smids_concurrent")
     return out.reshape(len(parts), n_ctas)
+
+
+def decode_profile(part: int, n_ctas: int) -> np.ndarray:
+    out = np.zeros(n_ctas * 8, dtype=np.uint64)
+    _check(lib().mx_decode_profile(part, out.ctypes.data_as(C.POINTER(C.c_uint64)), n_ctas * 8),
+           "mx_decode_profile")
+    return out.reshape(n_ctas, 8)
 
 
 def launch_count() -> int:

@@ -1,0 +1,50 @@
+"""Profiling driver: run GPT-2s (or another config) decode tasks on one partition.
+
+    python tools/prof_decode.py --sms 12 --tasks 2 [--cfg gpt2s] [--layers N]
+
+Used under ncu (`-k regex:decode_kernel -s 1 -c 1`) to capture one warm launch.
+"""
+import argparse
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_sc_dhakalrwercfm23_b200 import mx  # noqa: E402
+from workloads.configs import DECODE_CFGS  # noqa: E402
+from workloads.inputs import prompt_tokens  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--sms", type=int, default=12)
+ap.add_argument("--tasks", type=int, default=2)
+ap.add_argument("--cfg", default="gpt2s")
+ap.add_argument("--layers", type=int, default=0)
+ap.add_argument("--batch", type=int, default=1)
+ap.add_argument("--P", type=int, default=16)
+ap.add_argument("--G", type=int, default=32)
+a = ap.parse_args()
+cfg = DECODE_CFGS[a.cfg]
+if a.layers:
+    cfg = cfg.with_layers(a.layers)
+mx.mx_init([0])
+p = mx.part_create(0, a.sms, 24 << 30)
+fn = mx.fn_register(mx.decode_desc(cfg, max_batch=a.batch))
+mx.fn_load(fn, p)
+for k in range(a.tasks):
+    t = mx.decode_task(fn, prompt_tokens(k + 1, a.batch, a.P, cfg.vocab), a.G)
+    h0 = time.perf_counter()
+    mx.fn_submit(p, t)
+    r = mx.fn_wait(t)
+    print(f"task {k}: status {r['status']} kernel {r['kernel_ns'] / 1e6:.3f} ms "
+          f"wall {(time.perf_counter() - h0) * 1e3:.1f} ms")
+if os.environ.get("MX_DECODE_PROF") == "1":
+    n = mx.part_query(p)["n_ctas"]
+    pr = mx.decode_profile(p, n).astype(float)
+    names = ["total", "grid_barrier", "stage_input", "ring_wait(c0)", "gemv", "attention",
+             "producer_wait", "-"]
+    tot = pr[:, 0].mean()
+    for i, nm in enumerate(names[:7]):
+        print(f"  {nm:14s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
+              f"  min {pr[:, i].min() / 1e6:8.2f} max {pr[:, i].max() / 1e6:8.2f}")
+mx.part_destroy(p)
+mx.mx_shutdown()
