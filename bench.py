@@ -119,6 +119,17 @@ class ClockSampler:
 # GPU arm
 # ---------------------------------------------------------------------------
 
+def max_over_ranks(values, dist):
+    """Element-wise max of per-rank timings (host-side gloo collective; the
+    data path itself has no collective: tasks are independent replicas)."""
+    if not dist:
+        return [float(v) for v in values]
+    import torch
+    t = torch.tensor([float(v) for v in values], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return [float(v) for v in t]
+
+
 def make_layout(mx, gpu, n, kind):
     sizes = (LAYOUTS_FILL if kind == "fill" else LAYOUTS_EQUAL)[n]
     parts = [mx.part_create(gpu, s, QUOTA) for s in sizes]
@@ -210,11 +221,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
     s = summarize(all_res, args.steps)
     span = s["span_s"]
     wall = h1 - h0
-    if dist:
-        import torch
-        t = torch.tensor([span, wall], dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        span, wall = float(t[0]), float(t[1])
+    span, wall = max_over_ranks([span, wall], dist)
     for p in parts:
         mx.part_destroy(p)
     mx.mx_shutdown()

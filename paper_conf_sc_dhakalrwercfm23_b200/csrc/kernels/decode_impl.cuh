@@ -210,6 +210,28 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
       const int kind = phase_kind(k, L, p.fuse_att);
       if (kind == PH_ATT) continue;
       const Phase ph = make_phase(p, kind, k / pl);
+      // L2 prefetch of the small operands the consumers will need a few us from
+      // now (they are evicted by the weight stream between steps): the norm
+      // gain of this phase, and for QKV(l) the cached keys/values of layer l
+      // (this CTA's share) plus the RoPE row of step s.
+      {
+        const int layer = k / pl;
+        const uint16_t* lw = p.w_layers + (uint64_t)layer * p.layer_stride;
+        if (kind == PH_QKV) prefetch_l2(lw + p.off_gattn, (uint32_t)p.d * 2u);
+        if (kind == PH_GU) prefetch_l2(lw + p.off_gmlp, (uint32_t)p.d * 2u);
+        if (kind == PH_LM) prefetch_l2(p.g_final, (uint32_t)p.d * 2u);
+        if (kind == PH_QKV) {
+          if (layer == 0) prefetch_l2(p.rope_cs + (size_t)s * p.hd, (uint32_t)p.hd * 4u);
+          if (s > 0) {
+            const uint32_t bytes = (uint32_t)s * (uint32_t)p.hd * 2u;
+            for (int it = cta; it < p.B * p.Hkv; it += C) {
+              const size_t row0 = ((size_t)layer * p.B * p.Hkv + it) * p.max_seq * p.hd;
+              prefetch_l2(p.kc + row0, bytes);
+              prefetch_l2(p.vc + row0, bytes);
+            }
+          }
+        }
+      }
       int r0, r1;
       my_rows(ph.R, C, cta, k, &r0, &r1);
       for (int r = r0; r < r1; r += ph.TR) {
@@ -241,143 +263,165 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
 // Attention for one (sequence b, head h) item by one warp. Writes o_h either to
 // global o (separate ATT phase) or into the lane-permuted O-phase input in
 // shared memory (fused). `writer` selects the single writer of Kc/Vc[t].
+//
+// Latency-oriented: the cached keys/values of a block of KB positions are
+// loaded together with the current token's q/k/v (one round trip for t < KB),
+// then consumed with an online (running-max) softmax block by block. Lanes own
+// keys for the scores (LPK lanes per key) and dims for the output.
 // ---------------------------------------------------------------------------
-template <int B>
-__device__ __forceinline__ void attend(const DecodeParams& p, const Smem& sm, int layer, int t, int b, int h,
-                       bool writer, bool to_smem, int warp, int lane) {
-  const int Hkv = p.Hkv, hd = p.hd, half = hd / 2;
+template <int B, int HD>
+__device__ __forceinline__ void attend_hd(const DecodeParams& p, const Smem& sm, int layer, int t,
+                                          int b, int h, bool writer, bool to_smem, int warp,
+                                          int lane) {
+  constexpr int HALF = HD / 2;
+  constexpr int PPL = (HALF + 31) / 32;       // rope pairs per lane
+  constexpr int KB = (HD <= 64) ? 32 : 16;    // keys per block
+  constexpr int LPK = 32 / KB;                // lanes per key
+  constexpr int KSEG = HD / LPK;              // key elements per lane
+  constexpr int KV4 = KSEG / 8;               // 16-byte loads per lane per key
+  constexpr int DPL = HD / 32;                // output dims per lane
+  const int Hkv = p.Hkv;
   const int kvh = h / (p.H / Hkv);
   float* qs = sm.att + warp * 3 * kAttHd;
   float* ks = qs + kAttHd;
   float* vs = ks + kAttHd;
-  const float scale_div = sqrtf((float)hd);
+  const float scale_div = sqrtf((float)HD);
   const float* base = p.qkv + (size_t)b * p.qkv_rows;
-  const size_t cache_row0 = ((((size_t)layer * B + b) * Hkv + kvh) * p.max_seq) * hd;
+  const size_t cache_row0 = ((((size_t)layer * B + b) * Hkv + kvh) * p.max_seq) * HD;
   uint16_t* kcache = p.kc + cache_row0;
   uint16_t* vcache = p.vc + cache_row0;
-  for (int i = lane; i < half; i += 32) {
-    const float c = p.rope_cs[((size_t)t * half + i) * 2 + 0];
-    const float sn = p.rope_cs[((size_t)t * half + i) * 2 + 1];
-    const float q1 = base[h * hd + i], q2 = base[h * hd + i + half];
-    qs[i] = q1 * c - q2 * sn;
-    qs[i + half] = q2 * c + q1 * sn;
-    const float* kb = base + p.q_dim + kvh * hd;
-    const float k1 = kb[i], k2 = kb[i + half];
-    const uint16_t kb1 = f32_to_bf16_rne(k1 * c - k2 * sn);
-    const uint16_t kb2 = f32_to_bf16_rne(k2 * c + k1 * sn);
-    const float* vb = base + p.q_dim + p.kv_dim + kvh * hd;
-    const uint16_t vb1 = f32_to_bf16_rne(vb[i]);
-    const uint16_t vb2 = f32_to_bf16_rne(vb[i + half]);
-    ks[i] = bf16_bits_to_f32(kb1);
-    ks[i + half] = bf16_bits_to_f32(kb2);
-    vs[i] = bf16_bits_to_f32(vb1);
-    vs[i + half] = bf16_bits_to_f32(vb2);
-    if (writer) {
-      kcache[(size_t)t * hd + i] = kb1;
-      kcache[(size_t)t * hd + i + half] = kb2;
-      vcache[(size_t)t * hd + i] = vb1;
-      vcache[(size_t)t * hd + i + half] = vb2;
+  const int kslot = lane / LPK, kseg = (lane % LPK) * KSEG;
+
+  // --- block loads (independent of the current token) ---------------------
+  uint4 kr[KV4];
+  uint32_t vv[KB][(DPL + 1) / 2];
+  auto load_block = [&](int m) {
+    const int j = m * KB + kslot;
+#pragma unroll
+    for (int i = 0; i < KV4; ++i)
+      kr[i] = (j < t) ? *reinterpret_cast<const uint4*>(kcache + (size_t)j * HD + kseg + 8 * i)
+                      : make_uint4(0, 0, 0, 0);
+#pragma unroll
+    for (int jj = 0; jj < KB; ++jj) {
+      const int jk = m * KB + jj;
+      const uint16_t* src = vcache + (size_t)jk * HD + lane * DPL;
+      if (DPL == 4) {
+        uint2 v2 = make_uint2(0u, 0u);
+        if (jk < t) v2 = *reinterpret_cast<const uint2*>(src);
+        vv[jj][0] = v2.x;
+        vv[jj][(DPL + 1) / 2 - 1] = v2.y;
+      } else if (DPL == 2) {
+        vv[jj][0] = (jk < t) ? *reinterpret_cast<const uint32_t*>(src) : 0u;
+      } else {
+        vv[jj][0] = (jk < t) ? (uint32_t)*src : 0u;
+      }
+    }
+  };
+  load_block(0);
+
+  // --- current token: RoPE(q), RoPE(k) -> bf16, v -> bf16 --------------------
+#pragma unroll
+  for (int pi = 0; pi < PPL; ++pi) {
+    const int i = lane + 32 * pi;
+    if (i < HALF) {
+      const float c = p.rope_cs[((size_t)t * HALF + i) * 2 + 0];
+      const float sn = p.rope_cs[((size_t)t * HALF + i) * 2 + 1];
+      const float q1 = base[h * HD + i], q2 = base[h * HD + i + HALF];
+      const float* kb = base + p.q_dim + kvh * HD;
+      const float k1 = kb[i], k2 = kb[i + HALF];
+      const float* vb = base + p.q_dim + p.kv_dim + kvh * HD;
+      const float v1 = vb[i], v2 = vb[i + HALF];
+      qs[i] = q1 * c - q2 * sn;
+      qs[i + HALF] = q2 * c + q1 * sn;
+      const uint16_t kb1 = f32_to_bf16_rne(k1 * c - k2 * sn);
+      const uint16_t kb2 = f32_to_bf16_rne(k2 * c + k1 * sn);
+      const uint16_t vb1 = f32_to_bf16_rne(v1);
+      const uint16_t vb2 = f32_to_bf16_rne(v2);
+      ks[i] = bf16_bits_to_f32(kb1);
+      ks[i + HALF] = bf16_bits_to_f32(kb2);
+      vs[i] = bf16_bits_to_f32(vb1);
+      vs[i + HALF] = bf16_bits_to_f32(vb2);
+      if (writer) {
+        kcache[(size_t)t * HD + i] = kb1;
+        kcache[(size_t)t * HD + i + HALF] = kb2;
+        vcache[(size_t)t * HD + i] = vb1;
+        vcache[(size_t)t * HD + i + HALF] = vb2;
+      }
     }
   }
   __syncwarp();
-  // scores: lane owns keys j = lane + 32 m
-  float sc[kMaxSeqCap / 32];
-  float mx = -FLT_MAX;
+
+  // --- blocks with online softmax -------------------------------------------
+  float m_run = -FLT_MAX, l_run = 0.f;
+  float acc[DPL];
 #pragma unroll
-  for (int m = 0; m < kMaxSeqCap / 32; ++m) {
-    sc[m] = -FLT_MAX;
-    if (32 * m <= t) {
-      const int j = lane + 32 * m;
-      if (j <= t) {
-        float dot = 0.f;
-        if (j < t) {
-          const uint16_t* kr = kcache + (size_t)j * hd;
-          for (int e = 0; e < hd; e += 8) {
-            const uint4 kv = *reinterpret_cast<const uint4*>(kr + e);
-            float kf[8];
-            unpack8(kv, kf);
+  for (int d = 0; d < DPL; ++d) acc[d] = 0.f;
+  for (int m = 0; m * KB <= t; ++m) {
+    if (m > 0) load_block(m);
+    const int j = m * KB + kslot;
+    float dot = 0.f;
+    if (j < t) {
 #pragma unroll
-            for (int q = 0; q < 8; ++q) dot = fmaf(qs[e + q], kf[q], dot);
-          }
-        } else {
-          for (int e = 0; e < hd; ++e) dot = fmaf(qs[e], ks[e], dot);
-        }
-        sc[m] = dot / scale_div;
-        mx = fmaxf(mx, sc[m]);
+      for (int i = 0; i < KV4; ++i) {
+        float kf[8];
+        unpack8(kr[i], kf);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) dot = fmaf(qs[kseg + 8 * i + q], kf[q], dot);
       }
+    } else if (j == t) {
+#pragma unroll 8
+      for (int e = 0; e < KSEG; ++e) dot = fmaf(qs[kseg + e], ks[kseg + e], dot);
     }
-  }
-  mx = warp_max(mx);
-  float e[kMaxSeqCap / 32];
-  float lsum = 0.f;
+    if (LPK == 2) dot += __shfl_xor_sync(0xffffffffu, dot, 1);
+    const float sc = (j <= t) ? dot / scale_div : -FLT_MAX;
+    const float bm = warp_max(sc);
+    const float new_m = fmaxf(m_run, bm);
+    const float ej = (j <= t) ? expf(sc - new_m) : 0.f;
+    const float scale = expf(m_run - new_m);
+    const float bsum = warp_sum((lane % LPK) == 0 ? ej : 0.f);
+    l_run = l_run * scale + bsum;
 #pragma unroll
-  for (int m = 0; m < kMaxSeqCap / 32; ++m) {
-    const int j = lane + 32 * m;
-    e[m] = (32 * m <= t && j <= t) ? expf(sc[m] - mx) : 0.f;
-    lsum += e[m];
-  }
-  const float sum = warp_sum(lsum);
-  // output: lane owns dims [lane*dpl, lane*dpl + dpl), dpl = hd/32; the value
-  // rows of up to 16 keys are loaded together, then consumed in key order.
-  const int dpl = hd >> 5;
-  float acc[4] = {0.f, 0.f, 0.f, 0.f};
-  for (int m = 0; 32 * m <= t; ++m) {
-    float em = 0.f;
+    for (int d = 0; d < DPL; ++d) acc[d] *= scale;
 #pragma unroll
-    for (int mm = 0; mm < kMaxSeqCap / 32; ++mm)
-      if (mm == m) em = e[mm];
-    const int jcnt = min(32, t + 1 - 32 * m);
-    for (int jj0 = 0; jj0 < jcnt; jj0 += 8) {
-      uint2 vr[8];
+    for (int jj = 0; jj < KB; ++jj) {
+      const int jk = m * KB + jj;
+      const float e = __shfl_sync(0xffffffffu, ej, jj * LPK);
+      float v[4];
+      if (jk == t) {
 #pragma unroll
-      for (int jj = 0; jj < 8; ++jj) {
-        const int j = 32 * m + jj0 + jj;
-        vr[jj] = make_uint2(0u, 0u);
-        if (jj0 + jj < jcnt && j < t) {
-          const uint16_t* src = vcache + (size_t)j * hd + lane * dpl;
-          if (dpl == 4)
-            vr[jj] = *reinterpret_cast<const uint2*>(src);
-          else if (dpl == 2)
-            vr[jj].x = *reinterpret_cast<const uint32_t*>(src);
-          else
-            vr[jj].x = *src;
-        }
+        for (int d = 0; d < 4; ++d) v[d] = (d < DPL) ? vs[lane * DPL + d] : 0.f;
+      } else {
+        v[0] = __uint_as_float(vv[jj][0] << 16);
+        v[1] = __uint_as_float(vv[jj][0] & 0xffff0000u);
+        v[2] = __uint_as_float(vv[jj][(DPL + 1) / 2 - 1] << 16);
+        v[3] = __uint_as_float(vv[jj][(DPL + 1) / 2 - 1] & 0xffff0000u);
       }
 #pragma unroll
-      for (int jj = 0; jj < 8; ++jj) {
-        const int j = 32 * m + jj0 + jj;
-        const float ej = __shfl_sync(0xffffffffu, em, (jj0 + jj) & 31);
-        if (jj0 + jj < jcnt) {
-          float v[4];
-          if (j == t) {
-#pragma unroll
-            for (int i = 0; i < 4; ++i) v[i] = (i < dpl) ? vs[lane * dpl + i] : 0.f;
-          } else {
-            v[0] = __uint_as_float(vr[jj].x << 16);
-            v[1] = __uint_as_float(vr[jj].x & 0xffff0000u);
-            v[2] = __uint_as_float(vr[jj].y << 16);
-            v[3] = __uint_as_float(vr[jj].y & 0xffff0000u);
-          }
-#pragma unroll
-          for (int i = 0; i < 4; ++i)
-            if (i < dpl) acc[i] = fmaf(ej, v[i], acc[i]);
-        }
-      }
+      for (int d = 0; d < DPL; ++d) acc[d] = fmaf(e, v[d], acc[d]);
     }
+    m_run = new_m;
   }
   const int KP = round256(p.q_dim);
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    if (i < dpl) {
-      const int dd = lane * dpl + i;
-      const float o = acc[i] / sum;
-      if (to_smem)
-        sm.xin[xidx(b, h * hd + dd, KP)] = o;
-      else
-        p.o[(size_t)b * p.q_dim + h * hd + dd] = o;
-    }
+  for (int d = 0; d < DPL; ++d) {
+    const int dd = lane * DPL + d;
+    const float o = acc[d] / l_run;
+    if (to_smem)
+      sm.xin[xidx(b, h * HD + dd, KP)] = o;
+    else
+      p.o[(size_t)b * p.q_dim + h * HD + dd] = o;
   }
   __syncwarp();
+}
+
+template <int B>
+__device__ __forceinline__ void attend(const DecodeParams& p, const Smem& sm, int layer, int t,
+                                       int b, int h, bool writer, bool to_smem, int warp, int lane) {
+  switch (p.hd) {
+    case 32: attend_hd<B, 32>(p, sm, layer, t, b, h, writer, to_smem, warp, lane); break;
+    case 64: attend_hd<B, 64>(p, sm, layer, t, b, h, writer, to_smem, warp, lane); break;
+    default: attend_hd<B, 128>(p, sm, layer, t, b, h, writer, to_smem, warp, lane); break;
+  }
 }
 
 // Separate attention phase (large attention): items spread over all warps of all CTAs.
