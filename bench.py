@@ -10,7 +10,8 @@ P = 16 prompt + G = 32 greedy tokens per task, 700 tasks per closed batch
 One bench step = one closed batch of N_TASKS tasks submitted through the C ABI
 (fn_submit with host prompt buffers) and collected with fn_wait (host token
 buffers) on the chosen partition layout of each GPU. Before the timed run a
-short sweep measures the 1 / 2 / 4 / 7 / 14-partition layouts (D0 "fill").
+short sweep measures the 1 / 2 / 4 / 7 / 14-partition layouts (D0 "fill") and
+the finer 18 / 37-partition layouts (4-SM groups); the timed run uses the best.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--layout auto|1|2|4|7|14]
     python bench.py --impl reference      # the CPU oracle on a bounded sample
@@ -180,7 +181,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
 
     # --- partition sweep (Fig. 4 analog: 1 vs 2/4/7/14 partitions) ----------------
     sweep = []
-    sweep_tasks = 140
+    sweep_tasks = 148
     for n in (args.sweep if args.sweep else []):
         parts = make_layout(mx, gpu, n, "fill")
         load(parts)
@@ -341,7 +342,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="mx", choices=["mx", "reference"])
     ap.add_argument("--layout", default="auto")
-    ap.add_argument("--sweep", default="1,2,4,7,14",
+    ap.add_argument("--sweep", default="1,2,4,7,14,18,37",
                     help="comma list of partition counts for the pre-run sweep ('' = none)")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
     args = ap.parse_args()

@@ -21,6 +21,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libmx.so")
+EXTRA_DEFS = [d for d in os.environ.get("MX_DEFS", "").split() if d]   # variant builds (-DMX_...)
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
@@ -40,15 +41,18 @@ def headers():
             + glob.glob(os.path.join(CSRC, "kernels", "*.cuh")) + [os.path.join(ROOT, "include", "mx.h")])
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+def build(force: bool = False, verbose: bool = False, out: str | None = None,
+          build_dir: str | None = None) -> str:
+    lib = out or LIB
+    bdir = build_dir or BUILD
+    os.makedirs(bdir, exist_ok=True)
     hdr_mtime = max(os.path.getmtime(h) for h in headers())
     objs = []
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "-I", CSRC,
-              "-I", os.path.join(ROOT, "include")]
+              "-I", os.path.join(ROOT, "include")] + EXTRA_DEFS
     for src in sources():
         rel = os.path.relpath(src, CSRC).replace(os.sep, "_")
-        obj = os.path.join(BUILD, rel + ".o")
+        obj = os.path.join(bdir, rel + ".o")
         objs.append(obj)
         if (not force and os.path.exists(obj) and os.path.getmtime(obj) > os.path.getmtime(src)
                 and os.path.getmtime(obj) > hdr_mtime):
@@ -66,21 +70,23 @@ def build(force: bool = False, verbose: bool = False) -> str:
             raise RuntimeError(f"compile failed: {src}")
         if verbose and r.stderr:
             sys.stderr.write(r.stderr)
-    lib_mtime = os.path.getmtime(LIB) if os.path.exists(LIB) else 0
+    lib_mtime = os.path.getmtime(lib) if os.path.exists(lib) else 0
     if force or lib_mtime < max(os.path.getmtime(o) for o in objs):
-        cmd = [nvcc()] + ARCH + ["-shared", "-o", LIB] + objs + ["-lpthread", "-ldl", "-lrt"]
+        cmd = [nvcc()] + ARCH + ["-shared", "-o", lib] + objs + ["-lpthread", "-ldl", "-lrt"]
         if verbose:
             print(" ".join(cmd), flush=True)
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
             raise RuntimeError("link failed")
-    return LIB
+    return lib
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("-v", "--verbose", action="store_true")
+    ap.add_argument("--out", default=None, help="library path (variant builds)")
+    ap.add_argument("--build-dir", default=None)
     a = ap.parse_args()
-    print(build(a.force, a.verbose))
+    print(build(a.force, a.verbose, a.out, a.build_dir))

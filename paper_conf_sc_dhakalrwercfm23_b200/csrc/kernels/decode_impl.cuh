@@ -42,6 +42,13 @@ enum PhaseKind { PH_QKV = 0, PH_ATT = 1, PH_O = 2, PH_GU = 3, PH_DOWN = 4, PH_LM
 
 constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
 constexpr int kAttHd = 128;                 // max head_dim
+#ifdef MX_NO_SLEEP
+#define MX_FULL_WAIT(b, ph) mbar_try_wait(b, ph)
+#define MX_EMPTY_WAIT(b, ph) mbar_try_wait(b, ph)
+#else
+#define MX_FULL_WAIT(b, ph) mbar_try_wait_sleep(b, ph, 20000u)
+#define MX_EMPTY_WAIT(b, ph) mbar_try_wait_sleep(b, ph, 20000u)
+#endif
 constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
 
 struct Phase {
@@ -152,7 +159,7 @@ int decode_smem_bytes(int B, int kmax, int* n_stages) {
   const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;
-  if (ns > 6) ns = 6;
+  if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;
   if (n_stages) *n_stages = ns;
   if (ns < 2) return -1;
   return ns * per_stage + fixed;
@@ -239,7 +246,7 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
         // never abandons the stream: after a barrier timeout the consumers run
         // through the remaining phases without waiting, so every slot is freed.
         const long long tw = clock64();
-        while (!mbar_try_wait_sleep(&sm.empty[stage], phase_bit ^ 1u, 20000u)) {
+        while (!MX_EMPTY_WAIT(&sm.empty[stage], phase_bit ^ 1u)) {
         }
         wait_cyc += clock64() - tw;
         const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
@@ -256,7 +263,7 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
       }
     }
   }
-  if (p.prof) p.prof[cta * 8 + 6] = (unsigned long long)wait_cyc;
+  if (p.prof) p.prof[cta * 16 + 6] = (unsigned long long)wait_cyc;
 }
 
 // ---------------------------------------------------------------------------
@@ -584,7 +591,7 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
 // ---------------------------------------------------------------------------
 template <int B>
 struct RowsPerUnit {
-  static constexpr int value = (B <= 2) ? 4 : (B <= 4 ? 2 : 1);
+  static constexpr int value = (B == 1) ? MX_ROWS_B1 : (B <= 2) ? 4 : (B <= 4 ? 2 : 1);
 };
 
 template <int B, int NR, int NCH>
@@ -666,7 +673,7 @@ template <int B, int NR, int KIND>
 __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                               int k, int s,
                               int tid_c, uint32_t& stage, uint32_t& phase_bit, int n_stages,
-                              long long& wait_cyc) {
+                              long long& wait_cyc, long long& unit_cyc, long long& unit_cnt) {
   const int C = p.n_ctas, cta = blockIdx.x;
   const int warp = tid_c >> 5, lane = tid_c & 31;
   const int K = ph.K, KP = ph.KP, NC = ph.NC, NG = ph.NG;
@@ -691,13 +698,14 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
     // every warp observes the stage fill before releasing it (keeps the empty
     // barrier's arrival count per round exact)
     const long long tw = clock64();
-    while (!mbar_try_wait_sleep(&sm.full[stage], phase_bit, 20000u)) {
+    while (!MX_FULL_WAIT(&sm.full[stage], phase_bit)) {
     }
     wait_cyc += clock64() - tw;
     const uint16_t* wt = reinterpret_cast<const uint16_t*>(sm.ring + (size_t)stage * kStageBytes);
     float* red = sm.red + (size_t)stage * kMaxUnits * B;
     int* cnt = sm.cnt + stage * kMaxUnits;
     for (; u < units; u += kConsumerWarps) {
+      const long long tu = clock64();
       const int gi = (NG == 1) ? u : u / NG;   // output group within the tile
       const int g = u - gi * NG;
       const int j0 = gi * per;                 // first tile-local output of the unit
@@ -802,6 +810,8 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
           default: break;
         }
       }
+      unit_cyc += clock64() - tu;
+      ++unit_cnt;
     }
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.empty[stage]);
@@ -819,24 +829,25 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
 template <int B>
 __device__ __forceinline__ void gemv_phase(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                            int k, int s, int tid_c, uint32_t& stage,
-                                           uint32_t& phase_bit, int n_stages, long long& wait_cyc) {
+                                           uint32_t& phase_bit, int n_stages, long long& wait_cyc,
+                                           long long& unit_cyc, long long& unit_cnt) {
   constexpr int NR = RowsPerUnit<B>::value;
   constexpr int NRG = NR < 2 ? 2 : NR;   // GU units always hold gate/up pairs
   switch (ph.kind) {
     case PH_QKV:
-      gemv_phase_nr<B, NR, PH_QKV>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      gemv_phase_nr<B, NR, PH_QKV>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
     case PH_O:
-      gemv_phase_nr<B, NR, PH_O>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      gemv_phase_nr<B, NR, PH_O>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
     case PH_GU:
-      gemv_phase_nr<B, NRG, PH_GU>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      gemv_phase_nr<B, NRG, PH_GU>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
     case PH_DOWN:
-      gemv_phase_nr<B, NR, PH_DOWN>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      gemv_phase_nr<B, NR, PH_DOWN>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
     default:
-      gemv_phase_nr<B, NR, PH_LM>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc);
+      gemv_phase_nr<B, NR, PH_LM>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
   }
 }
@@ -868,7 +879,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
   const int pl = phases_per_layer(p.fuse_att);
   uint32_t stage = 0, phase_bit = 0;
   unsigned long long target = p.bar_base;
-  long long c_bar = 0, c_stage = 0, c_wait = 0, c_gemv = 0, c_att = 0;
+  long long c_bar = 0, c_stage = 0, c_wait = 0, c_gemv = 0, c_att = 0, c_unit = 0, c_units = 0;
   const long long t_begin = clock64();
   for (int s = 0; s < S; ++s) {
     const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
@@ -889,7 +900,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
           c_att += t1 - t0;
         else
           c_stage += t1 - t0;
-        gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait);
+        gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait, c_unit, c_units);
         const long long t2 = clock64();
         c_gemv += t2 - t1;
         t0 = t2;
@@ -900,13 +911,15 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     }
   }
   if (p.prof && tid_c == 0) {
-    unsigned long long* pr = p.prof + blockIdx.x * 8;
+    unsigned long long* pr = p.prof + blockIdx.x * 16;
     pr[0] = (unsigned long long)(clock64() - t_begin);
     pr[1] = (unsigned long long)c_bar;
     pr[2] = (unsigned long long)c_stage;
     pr[3] = (unsigned long long)c_wait;
     pr[4] = (unsigned long long)c_gemv;
     pr[5] = (unsigned long long)c_att;
+    pr[7] = (unsigned long long)c_unit;
+    pr[8] = (unsigned long long)c_units;
   }
   // final token (argmax of the last step)
   if (blockIdx.x == 0) {

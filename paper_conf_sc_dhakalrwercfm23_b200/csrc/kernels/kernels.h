@@ -6,8 +6,20 @@
 
 namespace mxk {
 
-constexpr int kStageBytes = 32768;      // one TMA bulk stage of weight rows
-constexpr int kConsumerWarps = 12;      // GEMV / attention warps per CTA
+#ifndef MX_STAGE_KB
+#define MX_STAGE_KB 32
+#endif
+#ifndef MX_CONSUMER_WARPS
+#define MX_CONSUMER_WARPS 12
+#endif
+#ifndef MX_MAX_STAGES
+#define MX_MAX_STAGES 6
+#endif
+#ifndef MX_ROWS_B1
+#define MX_ROWS_B1 4
+#endif
+constexpr int kStageBytes = MX_STAGE_KB * 1024;   // one TMA bulk stage of weight rows
+constexpr int kConsumerWarps = MX_CONSUMER_WARPS;   // GEMV / attention warps per CTA
 constexpr int kDecodeThreads = 32 * (kConsumerWarps + 1);  // + 1 producer (TMA) warp
 constexpr int kMaxUnits = 128;          // (row, 256-col chunk) work units per tile
 constexpr int kMaxCtas = 160;           // >= 148 SMs

@@ -14,7 +14,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmx.so")
+LIB_PATH = os.environ.get("MX_LIB") or os.path.join(_HERE, "libmx.so")
 
 MX_OK, MX_ENOENT, MX_EDEVICE, MX_ENOMEM, MX_EBUSY = 0, -2, -5, -12, -16
 MX_ENODEV, MX_EINVAL, MX_ENOSM, MX_ETIMEDOUT, MX_ESTATE = -19, -22, -28, -110, -125

@@ -22,10 +22,17 @@ ap.add_argument("--layers", type=int, default=0)
 ap.add_argument("--batch", type=int, default=1)
 ap.add_argument("--P", type=int, default=16)
 ap.add_argument("--G", type=int, default=32)
+ap.add_argument("--vocab", type=int, default=0)
+ap.add_argument("--dff", type=int, default=0)
 a = ap.parse_args()
 cfg = DECODE_CFGS[a.cfg]
 if a.layers:
     cfg = cfg.with_layers(a.layers)
+from dataclasses import replace  # noqa: E402
+if a.vocab:
+    cfg = replace(cfg, vocab=a.vocab)
+if a.dff:
+    cfg = replace(cfg, d_ff=a.dff)
 mx.mx_init([0])
 p = mx.part_create(0, a.sms, 24 << 30)
 fn = mx.fn_register(mx.decode_desc(cfg, max_batch=a.batch))
@@ -35,14 +42,18 @@ for k in range(a.tasks):
     h0 = time.perf_counter()
     mx.fn_submit(p, t)
     r = mx.fn_wait(t)
-    print(f"task {k}: status {r['status']} kernel {r['kernel_ns'] / 1e6:.3f} ms "
+    from oracle.cost import decode_task_bytes
+    gbs = decode_task_bytes(cfg, a.batch, a.P, a.G) / r['kernel_ns']
+    print(f"task {k}: status {r['status']} kernel {r['kernel_ns'] / 1e6:.3f} ms  {gbs:.1f} GB/s "
+          f"({gbs / mx.part_query(p)['n_ctas']:.1f} GB/s/SM) "
           f"wall {(time.perf_counter() - h0) * 1e3:.1f} ms")
 if os.environ.get("MX_DECODE_PROF") == "1":
     n = mx.part_query(p)["n_ctas"]
-    pr = mx.decode_profile(p, n).astype(float)
+    pr = mx.decode_profile(p, 2 * n).astype(float).reshape(n, 16)
     names = ["total", "grid_barrier", "stage_input", "ring_wait(c0)", "gemv", "attention",
              "producer_wait", "-"]
     tot = pr[:, 0].mean()
+    print(f"  unit latency (warp0) {pr[:, 7].sum() / max(pr[:, 8].sum(), 1):.0f} cyc over {pr[:, 8].mean():.0f} units/CTA")
     for i, nm in enumerate(names[:7]):
         print(f"  {nm:14s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
               f"  min {pr[:, i].min() / 1e6:8.2f} max {pr[:, i].max() / 1e6:8.2f}")

@@ -122,6 +122,9 @@ LAYOUTS_FILL = {
     4: [40, 36, 36, 36],
     7: [24, 24, 20, 20, 20, 20, 20],
     14: [12] * 9 + [8] * 5,
+    # finer than the paper's 1-4 processes / BASELINE's 14 (extra sweep points)
+    18: [8] * 18 + [4],
+    37: [4] * 37,
 }
 LAYOUTS_EQUAL = {
     1: [148],
