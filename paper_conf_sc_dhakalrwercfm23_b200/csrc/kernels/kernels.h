@@ -94,8 +94,12 @@ struct MpnnParams {
   float* out;                // [n_mol]
   unsigned long long* stamps;
   int n_ctas;
+  const int* tile_off;       // [n_tiles+1] first molecule of each <=128-atom tile
+  int n_tiles;
 };
 int mpnn_smem_bytes();
+// Greedy, deterministic packing of molecules into <=128-atom / <=512-bond tiles.
+int mpnn_pack_tiles(const int* atom_off, const int* edge_off, int n_mol, int* tile_off);
 int launch_mpnn(const MpnnParams& p, void* stream);
 
 uint64_t launch_counter();

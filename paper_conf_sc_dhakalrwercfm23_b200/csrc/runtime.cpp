@@ -443,9 +443,10 @@ static int alloc_mpnn_slot(Partition& p, FnInst& fi, Slot& s) {
   if ((rc = alloc_ptr(p, (M + 1) * 4, &s.edge_off))) return rc;
   if ((rc = alloc_ptr(p, NE * 6, &s.edges))) return rc;
   if ((rc = alloc_ptr(p, M * 4, &s.out))) return rc;
+  if ((rc = alloc_ptr(p, (M + 1) * 4, &s.tile_off))) return rc;
   if ((rc = alloc_ptr(p, 64, &s.stamps))) return rc;
   s.err = s.stamps + 16;
-  s.h_in_bytes = align_up((M + 1) * 4, 64) * 2 + align_up(NA, 64) + NE * 6 + 64;
+  s.h_in_bytes = align_up((M + 1) * 4, 64) * 3 + align_up(NA, 64) + align_up(NE * 6, 64) + 64;
   s.h_out_bytes = M * 4;
   if ((rc = host_alloc(s.h_in_bytes, &s.h_in))) return rc;
   if ((rc = host_alloc(s.h_out_bytes, &s.h_out))) return rc;
@@ -627,6 +628,10 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
       memcpy(h4, t->edges.data(), (size_t)t->n_edges * 6);
       CU_TRY(drv().cuMemcpyHtoDAsync(s.edges, h4, (size_t)t->n_edges * 6, st));
     }
+    // deterministic tile packing (host) -> device
+    int* h5 = reinterpret_cast<int*>(h3 + align_up(t->n_atoms, 64) + align_up((size_t)t->n_edges * 6, 64));
+    const int n_tiles = mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
+    CU_TRY(drv().cuMemcpyHtoDAsync(s.tile_off, h5, (size_t)(n_tiles + 1) * 4, st));
     const mx_mpnn_cfg& m = d.mpnn;
     const uint16_t* wb = reinterpret_cast<const uint16_t*>(fi->weights);
     mxk::MpnnParams k{};
@@ -650,6 +655,8 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.out = reinterpret_cast<float*>(s.out);
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
     k.n_ctas = e->n_ctas;
+    k.tile_off = reinterpret_cast<const int*>(s.tile_off);
+    k.n_tiles = n_tiles;
     CU_TRY(drv().cuEventRecord(ev[0], st));
     if (mxk::launch_mpnn(k, st)) {
       set_error("mpnn launch failed");
