@@ -15,6 +15,7 @@ import os
 import shutil
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
@@ -47,7 +48,7 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None,
     bdir = build_dir or BUILD
     os.makedirs(bdir, exist_ok=True)
     hdr_mtime = max(os.path.getmtime(h) for h in headers())
-    objs = []
+    objs, jobs = [], []
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "-I", CSRC,
               "-I", os.path.join(ROOT, "include")] + EXTRA_DEFS
     for src in sources():
@@ -58,18 +59,24 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None,
                 and os.path.getmtime(obj) > hdr_mtime):
             continue
         cmd = [nvcc()] + ARCH + common + ["-c", src, "-o", obj]
-        if src.endswith(".cu"):
-            cmd += ["-Xptxas", "-v"] if verbose else []
-        else:
-            cmd += ["-x", "cu"] if False else []
+        if verbose and src.endswith(".cu"):
+            cmd += ["-Xptxas", "-v"]
+        jobs.append((src, cmd))
+
+    def compile_one(job):
+        src, cmd = job
         if verbose:
             print(" ".join(cmd), flush=True)
-        r = subprocess.run(cmd, capture_output=True, text=True)
-        if r.returncode != 0:
-            sys.stderr.write(r.stdout + r.stderr)
-            raise RuntimeError(f"compile failed: {src}")
-        if verbose and r.stderr:
-            sys.stderr.write(r.stderr)
+        return src, subprocess.run(cmd, capture_output=True, text=True)
+
+    # translation units compile in parallel (the decode kernel is one TU per batch size)
+    with ThreadPoolExecutor(max_workers=max(1, min(len(jobs), os.cpu_count() or 1))) as ex:
+        for src, r in ex.map(compile_one, jobs):
+            if r.returncode != 0:
+                sys.stderr.write(r.stdout + r.stderr)
+                raise RuntimeError(f"compile failed: {src}")
+            if verbose and r.stderr:
+                sys.stderr.write(r.stderr)
     lib_mtime = os.path.getmtime(lib) if os.path.exists(lib) else 0
     if force or lib_mtime < max(os.path.getmtime(o) for o in objs):
         cmd = [nvcc()] + ARCH + ["-shared", "-o", lib] + objs + ["-lpthread", "-ldl", "-lrt"]

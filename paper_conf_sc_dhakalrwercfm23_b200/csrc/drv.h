@@ -51,6 +51,8 @@ namespace mx {
   X(cuMemGetInfo)                  \
   X(cuMemHostAlloc)                \
   X(cuMemFreeHost)                 \
+  X(cuMemHostGetDevicePointer)     \
+  X(cuStreamQuery)                 \
   X(cuLaunchKernel)                \
   X(cuKernelSetAttribute)          \
   X(cuGetErrorString)

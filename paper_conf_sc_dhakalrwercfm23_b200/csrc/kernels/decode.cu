@@ -1,2 +1,64 @@
-// Decode megakernel translation unit; the implementation lives in decode_impl.cuh.
-#include "decode_impl.cuh"
+// Decode megakernel: host-side helpers and the batch-size dispatch. The
+// kernel template lives in decode_impl.cuh and is instantiated once per batch
+// size in decode_b*.cu (separate translation units, compiled in parallel).
+#include <algorithm>
+
+#include "kernels.h"
+
+namespace mxk {
+
+
+__host__ __device__ inline int round256_h(int k) { return (k + 255) & ~255; }
+
+template <int B>
+int launch_b(const DecodeParams& p, void* stream);
+template <int B>
+int set_attrs_b(int device);
+
+int decode_smem_bytes(int B, int kmax, int* n_stages) {
+  const int fixed = B * round256_h(kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 + 8 * 4 +
+                    kConsumerWarps * 8 * 4 + 128;
+  const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
+  const int cap = 227 * 1024;
+  int ns = (cap - fixed) / per_stage;
+  if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;
+  if (n_stages) *n_stages = ns;
+  if (ns < 2) return -1;
+  return ns * per_stage + fixed;
+}
+
+int decode_fuse_attention(int B, int H, int hd) { return (B * H * hd <= 1024) ? 1 : 0; }
+
+uint64_t decode_barriers(int L, int P, int G, int fuse_att) {
+  const uint64_t S = (uint64_t)(P + G - 1);
+  return S * (uint64_t)(fuse_att ? 4 : 5) * (uint64_t)L + (uint64_t)G;   // phases_per_layer() x L + G LM phases
+}
+
+int launch_decode(const DecodeParams& p, void* stream) {
+  switch (p.B) {
+    case 1: return launch_b<1>(p, stream);
+    case 2: return launch_b<2>(p, stream);
+    case 3: return launch_b<3>(p, stream);
+    case 4: return launch_b<4>(p, stream);
+    case 5: return launch_b<5>(p, stream);
+    case 6: return launch_b<6>(p, stream);
+    case 7: return launch_b<7>(p, stream);
+    case 8: return launch_b<8>(p, stream);
+    default: return -4;
+  }
+}
+
+int decode_set_attrs(int device) {
+  int rc = 0;
+  rc |= set_attrs_b<1>(device);
+  rc |= set_attrs_b<2>(device);
+  rc |= set_attrs_b<3>(device);
+  rc |= set_attrs_b<4>(device);
+  rc |= set_attrs_b<5>(device);
+  rc |= set_attrs_b<6>(device);
+  rc |= set_attrs_b<7>(device);
+  rc |= set_attrs_b<8>(device);
+  return rc;
+}
+
+}  // namespace mxk

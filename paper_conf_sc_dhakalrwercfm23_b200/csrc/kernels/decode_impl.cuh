@@ -41,7 +41,7 @@ namespace mxk {
 enum PhaseKind { PH_QKV = 0, PH_ATT = 1, PH_O = 2, PH_GU = 3, PH_DOWN = 4, PH_LM = 5 };
 
 constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
-constexpr int kAttHd = 128;                 // max head_dim
+
 #ifdef MX_NO_SLEEP
 #define MX_FULL_WAIT(b, ph) mbar_try_wait(b, ph)
 #define MX_EMPTY_WAIT(b, ph) mbar_try_wait(b, ph)
@@ -153,25 +153,6 @@ __device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int B, int km
   return s;
 }
 
-int decode_smem_bytes(int B, int kmax, int* n_stages) {
-  const int fixed = B * round256(kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 + 8 * 4 +
-                    kConsumerWarps * 8 * 4 + 128;
-  const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
-  const int cap = 227 * 1024;
-  int ns = (cap - fixed) / per_stage;
-  if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;
-  if (n_stages) *n_stages = ns;
-  if (ns < 2) return -1;
-  return ns * per_stage + fixed;
-}
-
-int decode_fuse_attention(int B, int H, int hd) { return (B * H * hd <= 1024) ? 1 : 0; }
-
-uint64_t decode_barriers(int L, int P, int G, int fuse_att) {
-  const uint64_t S = (uint64_t)(P + G - 1);
-  return S * (uint64_t)phases_per_layer(fuse_att) * (uint64_t)L + (uint64_t)G;
-}
-
 // Device-wide barrier among all CTAs of the launch (consumer warps only; the
 // producer warp never waits on it). A 4 s timeout sets *err; afterwards every
 // barrier passes without waiting, so a failed launch still terminates.
@@ -204,7 +185,7 @@ __device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned lon
 // ---------------------------------------------------------------------------
 // Producer: stream this CTA's weight rows of every phase of every step.
 // ---------------------------------------------------------------------------
-__device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stages) {
+static __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stages) {
   const int C = p.n_ctas, cta = blockIdx.x, L = p.L;
   const int S = p.P + p.G - 1;
   const int pl = phases_per_layer(p.fuse_att);
@@ -483,7 +464,10 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
           best = v > best ? v : best;
         }
         tok = (int)argmax_key_index(best);
-        if (cta == 0) p.tokens[tid_c * p.G + (s - p.P)] = tok;
+        if (cta == 0) {
+          p.tokens[tid_c * p.G + (s - p.P)] = tok;
+          __threadfence_system();   // ordered before the completion flag
+        }
       }
       sm.tok[tid_c] = tok;
     }
@@ -930,14 +914,27 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         best = v > best ? v : best;
       }
       p.tokens[tid_c * p.G + (p.G - 1)] = (int)argmax_key_index(best);
+      __threadfence_system();
     }
     named_bar_sync(1, kNCT);
-    if (tid_c == 0) p.stamps[1] = globaltimer();
+    if (tid_c == 0) {
+      const unsigned long long t_end = globaltimer();
+      p.stamps[1] = t_end;
+      if (p.h_stamps) {
+        // every CTA passed the last grid barrier, so all outputs are final
+        volatile unsigned long long* h = p.h_stamps;
+        h[0] = p.stamps[0];
+        h[1] = t_end;
+        h[2] = (unsigned long long)(unsigned)ld_volatile_i32(p.err);
+        __threadfence_system();
+        h[3] = p.done_tag;
+      }
+    }
   }
 }
 
 template <int B>
-static int launch_b(const DecodeParams& p, void* stream) {
+int launch_b(const DecodeParams& p, void* stream) {
   const int kmax = max(max(p.d, p.q_dim), p.ff);
   int ns = 0;
   const int smem = decode_smem_bytes(B, kmax, &ns);
@@ -949,32 +946,16 @@ static int launch_b(const DecodeParams& p, void* stream) {
                        stream, args);
 }
 
-int launch_decode(const DecodeParams& p, void* stream) {
-  switch (p.B) {
-    case 1: return launch_b<1>(p, stream);
-    case 2: return launch_b<2>(p, stream);
-    case 3: return launch_b<3>(p, stream);
-    case 4: return launch_b<4>(p, stream);
-    case 5: return launch_b<5>(p, stream);
-    case 6: return launch_b<6>(p, stream);
-    case 7: return launch_b<7>(p, stream);
-    case 8: return launch_b<8>(p, stream);
-    default: return -4;
-  }
-}
-
-int decode_set_attrs(int device) {
-  const int cap = 227 * 1024;
-  int rc = 0;
-  rc |= set_max_smem(decode_kernel<1>, cap, device);
-  rc |= set_max_smem(decode_kernel<2>, cap, device);
-  rc |= set_max_smem(decode_kernel<3>, cap, device);
-  rc |= set_max_smem(decode_kernel<4>, cap, device);
-  rc |= set_max_smem(decode_kernel<5>, cap, device);
-  rc |= set_max_smem(decode_kernel<6>, cap, device);
-  rc |= set_max_smem(decode_kernel<7>, cap, device);
-  rc |= set_max_smem(decode_kernel<8>, cap, device);
-  return rc;
+template <int B>
+int set_attrs_b(int device) {
+  return set_max_smem(decode_kernel<B>, 227 * 1024, device);
 }
 
 }  // namespace mxk
+
+// One translation unit per batch size (parallel compilation).
+#define MX_DECODE_INSTANTIATE(B)                                      \
+  namespace mxk {                                                     \
+  template int launch_b<B>(const DecodeParams& p, void* stream);      \
+  template int set_attrs_b<B>(int device);                            \
+  }

@@ -21,6 +21,7 @@ namespace mxk {
 constexpr int kStageBytes = MX_STAGE_KB * 1024;   // one TMA bulk stage of weight rows
 constexpr int kConsumerWarps = MX_CONSUMER_WARPS;   // GEMV / attention warps per CTA
 constexpr int kDecodeThreads = 32 * (kConsumerWarps + 1);  // + 1 producer (TMA) warp
+constexpr int kAttHd = 128;             // max attention head_dim
 constexpr int kMaxUnits = 128;          // (row, 256-col chunk) work units per tile
 constexpr int kMaxCtas = 160;           // >= 148 SMs
 constexpr int kMaxSeqCap = 512;         // attention keeps <= 16 scores per lane
@@ -51,14 +52,18 @@ struct DecodeParams {
   unsigned long long* cand;  // [kMaxCtas][B] per-CTA argmax keys
   uint16_t* kc;              // [L][B][Hkv][max_seq][hd] bf16
   uint16_t* vc;
-  const int* prompt;         // [B][P]
-  int* tokens;               // [B][G]
+  const int* prompt;         // [B][P] (host-mapped)
+  int* tokens;               // [B][G] (host-mapped)
   float* logits;             // [G][B][V] or nullptr
   unsigned long long* bar;   // grid barrier counter (monotone across launches)
   unsigned long long bar_base;
   unsigned long long* stamps;  // [2] globaltimer start / end
   int* err;                  // 0 ok, 1 barrier timeout
   unsigned long long* prof;  // [n_ctas][8] cycle buckets (MX_DECODE_PROF=1) or nullptr
+  // host-mapped completion record: [0] start, [1] end, [2] err, [3] = done_tag,
+  // written last (after a system-scope fence) by CTA 0
+  unsigned long long* h_stamps;
+  unsigned long long done_tag;
 };
 
 // 1 if every CTA computes the whole attention itself (B*H*hd <= 1024).
@@ -91,11 +96,15 @@ struct MpnnParams {
   const uint8_t* atom_type;  // [n_atoms]
   const int* edge_off;       // [n_mol+1]
   const uint32_t* edges;     // packed mx_bond (6 B each) as raw bytes
-  float* out;                // [n_mol]
+  float* out;                // [n_mol] (host-mapped)
   unsigned long long* stamps;
   int n_ctas;
   const int* tile_off;       // [n_tiles+1] first molecule of each <=128-atom tile
   int n_tiles;
+  // host-mapped completion record (as DecodeParams), written by the last CTA to
+  // finish; stamps[4] is the CTA-completion counter (reset by that CTA)
+  unsigned long long* h_stamps;
+  unsigned long long done_tag;
 };
 int mpnn_smem_bytes();
 // Greedy, deterministic packing of molecules into <=128-atom / <=512-bond tiles.

@@ -336,12 +336,33 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         float part = 0.f;
         for (int f = lane; f < kF; f += 32) part = fmaf(bf16_bits_to_f32(p.w2[f]), z[f], part);
         part = warp_sum(part);
-        if (lane == 0) p.out[mb + warp] = part + bf16_bits_to_f32(p.c2[0]);
+        if (lane == 0) {
+          p.out[mb + warp] = part + bf16_bits_to_f32(p.c2[0]);
+          __threadfence_system();   // ordered before the completion flag
+        }
       }
       __syncthreads();
     }
   }
-  if (tid == 0) atomicMax(&p.stamps[1], (unsigned long long)globaltimer());
+  __syncthreads();
+  if (tid == 0) {
+    atomicMax(&p.stamps[1], (unsigned long long)globaltimer());
+    if (p.h_stamps) {
+      __threadfence_system();
+      // the last CTA to finish publishes the completion record
+      if (atomicAdd(&p.stamps[4], 1ull) == (unsigned long long)(gridDim.x - 1)) {
+        __threadfence();
+        volatile unsigned long long* st = p.stamps;
+        volatile unsigned long long* h = p.h_stamps;
+        h[0] = st[0];
+        h[1] = st[1];
+        h[2] = 0;
+        p.stamps[4] = 0;
+        __threadfence_system();
+        h[3] = p.done_tag;
+      }
+    }
+  }
 }
 
 int launch_mpnn(const MpnnParams& p, void* stream) {

@@ -313,11 +313,18 @@ static int alloc_ptr(Partition& p, uint64_t bytes, CUdeviceptr* out) {
   return rc;
 }
 
-static int host_alloc(size_t bytes, void** out) {
+// Pinned, portable, device-mapped host memory; *dev = its device address.
+static int host_alloc(size_t bytes, void** out, CUdeviceptr* dev = nullptr) {
   if (bytes == 0) bytes = 64;
-  if (drv().cuMemHostAlloc(out, bytes, CU_MEMHOSTALLOC_PORTABLE) != CUDA_SUCCESS) {
+  if (drv().cuMemHostAlloc(out, bytes, CU_MEMHOSTALLOC_PORTABLE | CU_MEMHOSTALLOC_DEVICEMAP) !=
+      CUDA_SUCCESS) {
     set_error("pinned host allocation of %zu bytes failed", bytes);
     return MX_ENOMEM;
+  }
+  memset(*out, 0, bytes);
+  if (dev && drv().cuMemHostGetDevicePointer(dev, *out, 0) != CUDA_SUCCESS) {
+    set_error("mapping pinned host memory into the device address space failed");
+    return MX_EDEVICE;
   }
   return MX_OK;
 }
@@ -428,9 +435,9 @@ static int alloc_decode_slot(Partition& p, FnInst& fi, Slot& s) {
   s.err = s.stamps + 16;
   s.h_in_bytes = B * T * 4;
   s.h_out_bytes = B * T * 4 + T * B * V * 4;
-  if ((rc = host_alloc(s.h_in_bytes, &s.h_in))) return rc;
-  if ((rc = host_alloc(s.h_out_bytes, &s.h_out))) return rc;
-  if ((rc = host_alloc(64, reinterpret_cast<void**>(&s.h_stamps)))) return rc;
+  if ((rc = host_alloc(s.h_in_bytes, &s.h_in, &s.d_in))) return rc;
+  if ((rc = host_alloc(s.h_out_bytes, &s.h_out, &s.d_out))) return rc;
+  if ((rc = host_alloc(64, reinterpret_cast<void**>(&s.h_stamps), &s.d_stamps))) return rc;
   return MX_OK;
 }
 
@@ -448,9 +455,9 @@ static int alloc_mpnn_slot(Partition& p, FnInst& fi, Slot& s) {
   s.err = s.stamps + 16;
   s.h_in_bytes = align_up((M + 1) * 4, 64) * 3 + align_up(NA, 64) + align_up(NE * 6, 64) + 64;
   s.h_out_bytes = M * 4;
-  if ((rc = host_alloc(s.h_in_bytes, &s.h_in))) return rc;
-  if ((rc = host_alloc(s.h_out_bytes, &s.h_out))) return rc;
-  if ((rc = host_alloc(64, reinterpret_cast<void**>(&s.h_stamps)))) return rc;
+  if ((rc = host_alloc(s.h_in_bytes, &s.h_in, &s.d_in))) return rc;
+  if ((rc = host_alloc(s.h_out_bytes, &s.h_out, &s.d_out))) return rc;
+  if ((rc = host_alloc(64, reinterpret_cast<void**>(&s.h_stamps), &s.d_stamps))) return rc;
   return MX_OK;
 }
 
@@ -546,11 +553,19 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     s.need_reset = false;
   }
   const mx_fn_desc& d = fi->fn->desc;
+  // Completion: the kernel writes its results and a done tag into host-mapped
+  // memory, so a task is ONE kernel launch in the stream with nothing queued
+  // behind it (copies / event records after a kernel would block unrelated
+  // partitions' streams that share its hardware channel). Parity mode
+  // (logits requested) keeps a D2H copy and an event.
+  t->use_flag = !(t->kind == MX_FN_DECODE && t->out_logits);
+  t->polls = 0;
+  volatile uint64_t* hst = s.h_stamps;
+  hst[3] = 0;
   if (t->kind == MX_FN_DECODE) {
     const mx_decode_cfg& c = d.dec;
     const size_t pb = (size_t)t->B * t->P * 4;
-    memcpy(s.h_in, t->prompt.data(), pb);
-    CU_TRY(drv().cuMemcpyHtoDAsync(s.prompt, s.h_in, pb, st));
+    memcpy(s.h_in, t->prompt.data(), pb);   // read by the kernel through the mapping
     mxk::DecodeParams k{};
     k.L = c.n_layers;
     k.d = c.d_model;
@@ -590,27 +605,28 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.cand = reinterpret_cast<unsigned long long*>(s.cand);
     k.kc = reinterpret_cast<uint16_t*>(s.kc);
     k.vc = reinterpret_cast<uint16_t*>(s.vc);
-    k.prompt = reinterpret_cast<const int*>(s.prompt);
-    k.tokens = reinterpret_cast<int*>(s.tokens);
+    k.prompt = reinterpret_cast<const int*>(s.d_in);
+    k.tokens = reinterpret_cast<int*>(s.d_out);
+    k.h_stamps = reinterpret_cast<unsigned long long*>(s.d_stamps);
+    k.done_tag = t->id;
     k.logits = t->out_logits ? reinterpret_cast<float*>(s.logits) : nullptr;
     k.bar = reinterpret_cast<unsigned long long*>(s.bar);
     k.bar_base = s.bar_count;
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
     k.err = reinterpret_cast<int*>(s.err);
     k.prof = g_decode_prof ? reinterpret_cast<unsigned long long*>(p.sys + 65536) : nullptr;
-    CU_TRY(drv().cuEventRecord(ev[0], st));
+    if (!t->use_flag) CU_TRY(drv().cuEventRecord(ev[0], st));
     int rc = mxk::launch_decode(k, st);
     if (rc) {
       set_error("decode launch failed (%d)", rc);
       return MX_EDEVICE;
     }
-    CU_TRY(drv().cuEventRecord(ev[1], st));
     s.bar_count += mxk::decode_barriers(k.L, k.P, k.G, k.fuse_att) * (uint64_t)k.n_ctas;
-    const size_t tb = (size_t)t->B * t->G * 4;
-    CU_TRY(drv().cuMemcpyDtoHAsync(s.h_out, s.tokens, tb, st));
-    if (t->out_logits)
+    if (!t->use_flag) {
+      CU_TRY(drv().cuEventRecord(ev[1], st));
       CU_TRY(drv().cuMemcpyDtoHAsync(static_cast<uint8_t*>(s.h_out) + (size_t)t->B * c.max_seq * 4,
                                      s.logits, (size_t)t->G * t->B * c.vocab * 4, st));
+    }
   } else {
     // pack CSR inputs into pinned staging, one H2D per array
     uint8_t* h = static_cast<uint8_t*>(s.h_in);
@@ -652,32 +668,44 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.atom_type = reinterpret_cast<const uint8_t*>(s.atom_type);
     k.edge_off = reinterpret_cast<const int*>(s.edge_off);
     k.edges = reinterpret_cast<const uint32_t*>(s.edges);
-    k.out = reinterpret_cast<float*>(s.out);
+    k.out = reinterpret_cast<float*>(s.d_out);
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
+    k.h_stamps = reinterpret_cast<unsigned long long*>(s.d_stamps);
+    k.done_tag = t->id;
     k.n_ctas = e->n_ctas;
     k.tile_off = reinterpret_cast<const int*>(s.tile_off);
     k.n_tiles = n_tiles;
-    CU_TRY(drv().cuEventRecord(ev[0], st));
     if (mxk::launch_mpnn(k, st)) {
       set_error("mpnn launch failed");
       return MX_EDEVICE;
     }
-    CU_TRY(drv().cuEventRecord(ev[1], st));
-    CU_TRY(drv().cuMemcpyDtoHAsync(s.h_out, s.out, (size_t)t->n_mol * 4, st));
   }
-  CU_TRY(drv().cuMemcpyDtoHAsync(s.h_stamps, s.stamps, 24, st));
-  CU_TRY(drv().cuEventRecord(ev[2], st));
+  if (!t->use_flag) {
+    CU_TRY(drv().cuMemcpyDtoHAsync(s.h_stamps, s.stamps, 24, st));
+    CU_TRY(drv().cuEventRecord(ev[2], st));
+  }
   e->inflight++;
   return MX_OK;
+}
+
+static bool task_flag_seen(const Task* t) {
+  const volatile uint64_t* st = t->inst->slots[t->slot].h_stamps;
+  if (st[3] != t->id) return false;
+  std::atomic_thread_fence(std::memory_order_acquire);
+  return true;
 }
 
 static void finish_task(Gpu& gpu, Task* t, bool dev_ok) {
   Slot& s = t->inst->slots[t->slot];
   Exec* e = t->exec;
+  const volatile uint64_t* st = s.h_stamps;
   float ms = 0.f;
-  if (dev_ok && drv().cuEventElapsedTime(&ms, e->ev[t->lane][0], e->ev[t->lane][1]) == CUDA_SUCCESS)
-    t->kernel_ns = (uint64_t)((double)ms * 1e6);
-  const uint64_t* st = s.h_stamps;
+  if (!t->use_flag) {
+    if (dev_ok && drv().cuEventElapsedTime(&ms, e->ev[t->lane][0], e->ev[t->lane][1]) == CUDA_SUCCESS)
+      t->kernel_ns = (uint64_t)((double)ms * 1e6);
+  } else if (dev_ok && st[1] >= st[0]) {
+    t->kernel_ns = st[1] - st[0];   // device %globaltimer span of the launch
+  }
   const int err = dev_ok ? (int)(st[2] & 0xffffffffu) : 1;
   t->status = (!dev_ok || err) ? MX_EDEVICE : MX_OK;
   if (t->kind == MX_FN_DECODE) {
@@ -697,6 +725,26 @@ static void finish_task(Gpu& gpu, Task* t, bool dev_ok) {
   e->inflight--;
 }
 
+// Tasks kept in flight per partition. Two (double-buffered task slots) hide
+// the host reaction time between consecutive tasks, but every queued-behind
+// kernel occupies its hardware channel: once a GPU has more partition streams
+// than CUDA_DEVICE_MAX_CONNECTIONS (32) can give their own channel, a second
+// queued task blocks the unrelated streams sharing that channel until the
+// first one ends (measured: 37 partitions, busy fraction 0.78 -> one-task
+// gaps). So more than kDeepPartsMax partitions per GPU run one task at a
+// time (the host reaction, ~10s of us, is < 0.1% of a decode task).
+// MX_INFLIGHT=1|2 overrides.
+static constexpr size_t kDeepPartsMax = 16;
+static size_t g_inflight_override = 0;
+
+static size_t inflight_depth(const Gpu& gpu) {
+  if (g_inflight_override) return g_inflight_override;
+  size_t live = 0;
+  for (const Partition* p : gpu.parts)
+    if (p->live) ++live;
+  return live > kDeepPartsMax ? 1 : 2;
+}
+
 static void dispatcher_main(Lib* L, Gpu* gpu) {
   drv().cuCtxSetCurrent(gpu->primary);
   std::vector<Task*> completed;
@@ -706,17 +754,37 @@ static void dispatcher_main(Lib* L, Gpu* gpu) {
     {
       std::unique_lock<std::mutex> lk(gpu->mu);
       bool progress = false;
+      const size_t depth = inflight_depth(*gpu);
       for (Partition* p : gpu->parts) {
         while (!p->inflight.empty()) {
           Task* t = p->inflight.front();
-          CUresult r = drv().cuEventQuery(t->exec->ev[t->lane][2]);
-          if (r == CUDA_ERROR_NOT_READY) break;
-          finish_task(*gpu, t, r == CUDA_SUCCESS);
+          bool ok = true;
+          if (t->use_flag) {
+            if (!task_flag_seen(t)) {
+              // no flag yet: every 256th poll ask the driver whether the stream
+              // faulted (or drained without the kernel signalling)
+              if ((++t->polls & 255u) != 0) break;
+              CUresult r = drv().cuStreamQuery(t->exec->stream);
+              if (r == CUDA_ERROR_NOT_READY) break;
+              if (r == CUDA_SUCCESS && !task_flag_seen(t)) {
+                // the stream is idle only after the kernel ended: its flag must be there
+                if ((t->polls >> 8) < 4) break;   // allow the PCIe write to land
+                set_error("task %llu: kernel ended without its completion flag",
+                          (unsigned long long)t->id);
+              }
+              ok = (r == CUDA_SUCCESS) && task_flag_seen(t);
+            }
+          } else {
+            CUresult r = drv().cuEventQuery(t->exec->ev[t->lane][2]);
+            if (r == CUDA_ERROR_NOT_READY) break;
+            ok = (r == CUDA_SUCCESS);
+          }
+          finish_task(*gpu, t, ok);
           p->inflight.pop_front();
           completed.push_back(t);
           progress = true;
         }
-        while (p->inflight.size() < 2 && !p->fifo.empty() && p->fifo.front()->ready) {
+        while (p->inflight.size() < depth && !p->fifo.empty() && p->fifo.front()->ready) {
           Task* t = p->fifo.front();
           p->fifo.pop_front();
           if (launch_task(*gpu, *p, t) != MX_OK) {
@@ -854,6 +922,10 @@ static int init_impl(const std::vector<int>& ordinals) {
   if (g_lib) return MX_OK;
   setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
   g_decode_prof = getenv("MX_DECODE_PROF") && atoi(getenv("MX_DECODE_PROF")) == 1;
+  if (const char* e = getenv("MX_INFLIGHT")) {
+    const int v = atoi(e);
+    g_inflight_override = (v == 1 || v == 2) ? (size_t)v : 0;
+  }
   const char* why = nullptr;
   if (!drv().load(&why)) {
     set_error("%s (no CUDA driver?)", why ? why : "driver load failed");

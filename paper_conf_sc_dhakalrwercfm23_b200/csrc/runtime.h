@@ -65,6 +65,8 @@ struct Task {
   int slot = -1;
   Exec* exec = nullptr;
   int lane = 0;
+  bool use_flag = false;      // completion = kernel-written host flag (no stream events)
+  uint32_t polls = 0;
   // completion
   mx_status status = MX_OK;
   bool done = false;
@@ -89,7 +91,10 @@ struct Slot {
   size_t h_in_bytes = 0;
   void* h_out = nullptr;
   size_t h_out_bytes = 0;
-  uint64_t* h_stamps = nullptr;   // [2] + err word
+  uint64_t* h_stamps = nullptr;   // [0] start, [1] end, [2] err, [3] done tag (host-mapped)
+  // device views of the host-mapped buffers (kernels write results and the
+  // completion flag there directly; no copy-engine work in the stream)
+  CUdeviceptr d_in = 0, d_out = 0, d_stamps = 0;
 };
 
 struct Fn {

@@ -45,3 +45,37 @@ def summarize(results, n_generated_tokens: int, algo_bytes: int, peak_gbs: float
         out["hbm_gbs"] = algo_bytes / dev_span * 1e-9
         out["hbm_frac"] = out["hbm_gbs"] / peak_gbs
     return out
+
+
+def decode_task_bytes(cfg, B: int, P: int, G: int) -> int:
+    """Algorithmic HBM bytes of one greedy decode task (SURVEY.md §8(d) D0,
+    DESIGN.md §6): every weight once per step (LM head only at the G steps that
+    produce a token), the embedding row, and the KV cache read/written."""
+    d, q, kv, ff = cfg.d_model, cfg.q_dim, cfg.kv_dim, cfg.d_ff
+    layer = 2 * (d * q + 2 * d * kv + q * d + 3 * d * ff) + 4 * d
+    head = 2 * cfg.vocab * d + 2 * d
+    S = P + G - 1
+    kvpos = cfg.n_layers * 2 * kv * 2
+    return (S * cfg.n_layers * layer + G * head + S * B * 2 * d + B * kvpos * (S * (S + 1) // 2)
+            + S * B * kvpos)
+
+
+def mpnn_task_flops(task: dict, F: int, T: int) -> int:
+    """Algorithmic flops of one MPNN task, summed over its
+    molecules: T*(2F^2*(n + D_ub) + E_dir*F + 2n*F) + n*F + 2F^2 + 4F, with
+    D_ub the number of distinct (atom, incident bond type) pairs."""
+    ao = np.asarray(task["atom_off"], dtype=np.int64)
+    eo = np.asarray(task["edge_off"], dtype=np.int64)
+    e = task["edges"]
+    M = len(ao) - 1
+    n = np.diff(ao)
+    E = np.diff(eo)
+    mol_of_edge = np.repeat(np.arange(M), E)
+    base = ao[:-1][mol_of_edge]
+    b = e["bond"].astype(np.int64)
+    gu = (base + e["u"].astype(np.int64)) * 4 + b
+    gv = (base + e["v"].astype(np.int64)) * 4 + b
+    D = len(np.unique(np.concatenate([gu, gv])))
+    tot_n, tot_E = int(n.sum()), int(E.sum())
+    return int(T * (2 * F * F * (tot_n + D) + 2 * tot_E * F + 2 * tot_n * F) + tot_n * F
+               + M * (2 * F * F + 4 * F))

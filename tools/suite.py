@@ -1,0 +1,330 @@
+#!/usr/bin/env python3
+"""Measurement suite for the SURVEY.md §8(d) rows beyond the headline bench
+(bench.py = D2, configs[1]). Each subcommand prints ONE JSON line.
+
+    python tools/suite.py smsweep   # D2b: single-instance SM sweep (Fig. 2 analog)
+    python tools/suite.py c3        # D3:  7B-Llama-shaped decode, B 1/2/4/8, 1/2/4 partitions, 14 GiB quotas
+    python tools/suite.py c4        # D4:  decode + MPNN co-located on 7 partitions vs 1 (WLAW)
+    python tools/suite.py c5        # D5:  10k-task farm, 50/50 mix, part_resize every 1000 submissions
+    python tools/suite.py modes     # N1:  partitioned vs unpartitioned-concurrent vs time-shared
+
+All inputs are seeded and synthetic (workloads/); weights are generated on the
+device from seeds. Times are device %globaltimer stamps (t_start/t_end of each
+task); HBM fractions use algorithmic bytes (metrics.decode_task_bytes) over the
+device span against MEASURED_PEAKS.json. Output parity of these workloads is
+covered by tests/ (-m gpu); this tool only measures.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from paper_conf_sc_dhakalrwercfm23_b200.metrics import (decode_task_bytes,  # noqa: E402
+                                                        mpnn_task_flops, percentiles)
+from workloads.configs import GPT2S, LLAMA7B, MPNN, LAYOUTS_FILL  # noqa: E402
+from workloads.inputs import molecules, prompt_tokens, shuffle  # noqa: E402
+
+P_LEN, G_LEN = 16, 32
+MOLS = 1024
+
+
+def peak_gbs():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"])
+    except Exception:
+        return 6650.0
+
+
+def peak_bf16_tflops():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        for k in ("bf16_tflops", "bf16_dense_tflops", "tc_bf16_tflops"):
+            if k in d:
+                return float(d[k])
+    except Exception:
+        pass
+    return 2250.0
+
+
+def closed_batch(mx, items):
+    """items: list of (part_or_ANY, Task). Submit all at t0, wait all.
+    Returns (results, host wall seconds)."""
+    h0 = time.perf_counter()
+    for part, t in items:
+        mx.fn_submit(part, t)
+    res = [mx.fn_wait(t) for _, t in items]
+    wall = time.perf_counter() - h0
+    bad = [r for r in res if r["status"] != 0]
+    if bad:
+        raise RuntimeError(f"{len(bad)} task(s) failed, first {bad[0]}")
+    return res, wall
+
+
+def span_s(res):
+    return (max(r["t_end_ns"] for r in res) - min(r["t_start_ns"] for r in res)) / 1e9
+
+
+def lat(res):
+    comp = [(r["t_end_ns"] - r["t_submit_ns"]) / 1e6 for r in res]
+    serv = [(r["t_end_ns"] - r["t_start_ns"]) / 1e6 for r in res]
+    c, s = percentiles(comp), percentiles(serv)
+    return {"p50_ms": round(c["p50"], 3), "p99_ms": round(c["p99"], 3),
+            "service_p50_ms": round(s["p50"], 3), "service_p99_ms": round(s["p99"], 3)}
+
+
+# ---------------------------------------------------------------------------
+# D2b: single instance, SM sweep
+# ---------------------------------------------------------------------------
+
+def cmd_smsweep(a, mx):
+    cfg = GPT2S
+    fn = mx.fn_register(mx.decode_desc(cfg))
+    bytes_task = decode_task_bytes(cfg, 1, P_LEN, G_LEN)
+    steps = P_LEN + G_LEN - 1
+    rows = []
+    for sm in [int(x) for x in a.sms.split(",")]:
+        p = mx.part_create(0, sm, 512 << 20)
+        got = mx.part_query(p)["sm_count"]
+        mx.fn_load(fn, p)
+        warm = mx.decode_task(fn, prompt_tokens(1, 1, P_LEN, cfg.vocab), G_LEN)
+        closed_batch(mx, [(p, warm)])
+        items = [(p, mx.decode_task(fn, prompt_tokens(k, 1, P_LEN, cfg.vocab), G_LEN))
+                 for k in range(1, a.tasks + 1)]
+        res, _ = closed_batch(mx, items)
+        kern = float(np.median([r["kernel_ns"] for r in res])) / 1e9
+        rows.append({"sm": got, "task_ms": round(kern * 1e3, 3),
+                     "step_us": round(kern / steps * 1e6, 2),
+                     "gbs": round(bytes_task / kern / 1e9, 1),
+                     "gbs_per_sm": round(bytes_task / kern / 1e9 / got, 2),
+                     "hbm_frac": round(bytes_task / kern / 1e9 / peak_gbs(), 4)})
+        mx.part_destroy(p)
+    return {"suite": "D2b smsweep", "workload": "configs[1] GPT-2s decode B=1 P=16 G=32, one "
+            "instance alone on a partition of `sm` SMs", "tasks_per_point": a.tasks,
+            "peak_gbs": peak_gbs(), "points": rows}
+
+
+# ---------------------------------------------------------------------------
+# D3: 7B-shaped decode, quotas
+# ---------------------------------------------------------------------------
+
+def cmd_c3(a, mx):
+    cfg = LLAMA7B
+    quota = 14 << 30
+    fn = mx.fn_register(mx.decode_desc(cfg, max_batch=8))
+    # negative: a 12 GiB quota cannot hold 12.55 GiB of weights (D3)
+    pn = mx.part_create(0, 8, 12 << 30)
+    try:
+        mx.fn_load(fn, pn)
+        enomem = "loaded (unexpected)"
+    except mx.MxError as e:
+        enomem = "MX_ENOMEM" if e.code == mx.MX_ENOMEM else f"error {e.code}"
+    mx.part_destroy(pn)
+    out_rows = []
+    batches = [int(x) for x in a.batches.split(",")]
+    for n in [int(x) for x in a.layouts.split(",")]:
+        sizes = LAYOUTS_FILL[n]
+        parts = [mx.part_create(0, s, quota) for s in sizes]
+        t0 = time.perf_counter()
+        for p in parts:
+            mx.fn_load(fn, p)
+        load_s = time.perf_counter() - t0
+        info = [mx.part_query(p) for p in parts]
+        for B in batches:
+            warm = [(p, mx.decode_task(fn, prompt_tokens(9000 + i, B, P_LEN, cfg.vocab), 2))
+                    for i, p in enumerate(parts)]
+            closed_batch(mx, warm)
+            items = []
+            for k in range(1, a.tasks + 1):
+                part = parts[(k - 1) % len(parts)]   # STATIC (k-1) mod P
+                items.append((part, mx.decode_task(fn, prompt_tokens(k, B, P_LEN, cfg.vocab),
+                                                   G_LEN)))
+            res, wall = closed_batch(mx, items)
+            sp = span_s(res)
+            tb = decode_task_bytes(cfg, B, P_LEN, G_LEN)
+            gbs = a.tasks * tb / sp / 1e9
+            out_rows.append({"partitions": n, "sms": sizes, "batch": B, "tasks": a.tasks,
+                             "tasks_per_s": round(a.tasks / sp, 4),
+                             "gen_tok_per_s": round(a.tasks * B * G_LEN / sp, 1),
+                             "hbm_gbs": round(gbs, 1), "hbm_frac": round(gbs / peak_gbs(), 4),
+                             **lat(res)})
+        out_rows[-1]["load_s_all_partitions"] = round(load_s, 3)
+        out_rows[-1]["hbm_peak_bytes"] = [i["hbm_peak"] for i in info]
+        for p in parts:
+            mx.part_destroy(p)
+    for r in out_rows:
+        base = [x for x in out_rows if x["partitions"] == 1 and x["batch"] == r["batch"]]
+        if base:
+            r["ratio_vs_1_partition"] = round(r["tasks_per_s"] / base[0]["tasks_per_s"], 3)
+    return {"suite": "D3 c3", "workload": "configs[2] 7B-Llama-shaped decode (L32 d4096 "
+            "d_ff11008 V32000), P=16 G=32, STATIC placement, quota 14 GiB per partition",
+            "quota_12GiB_fn_load": enomem, "peak_gbs": peak_gbs(), "rows": out_rows}
+
+
+# ---------------------------------------------------------------------------
+# D4 / D5: mixed decode + MPNN
+# ---------------------------------------------------------------------------
+
+def mixed_items(mx, fd, fm, n_dec, n_mpnn, mol_cache):
+    kinds = shuffle([("d", k) for k in range(1, n_dec + 1)] +
+                    [("m", k) for k in range(1, n_mpnn + 1)], 42)
+    items = []
+    for kind, k in kinds:
+        if kind == "d":
+            items.append(("d", mx.decode_task(fd, prompt_tokens(k, 1, P_LEN, GPT2S.vocab), G_LEN)))
+        else:
+            mol = mol_cache[(k - 1) % len(mol_cache)]
+            items.append(("m", mx.mpnn_task(fm, mol)))
+    return items
+
+
+def class_stats(res, kinds, mflops_mean, n_dec, n_mpnn):
+    out = {}
+    sp = span_s(res)
+    for c, name in (("d", "decode"), ("m", "mpnn")):
+        rr = [r for r, k in zip(res, kinds) if k == c]
+        if not rr:
+            continue
+        s = lat(rr)
+        s["tasks_per_s"] = round(len(rr) / sp, 3)
+        out[name] = s
+    dec_bytes = n_dec * decode_task_bytes(GPT2S, 1, P_LEN, G_LEN)
+    out["decode_hbm_frac"] = round(dec_bytes / sp / 1e9 / peak_gbs(), 4)
+    out["mpnn_tflops"] = round(n_mpnn * mflops_mean / sp / 1e12, 2)
+    out["mpnn_tc_frac"] = round(out["mpnn_tflops"] / peak_bf16_tflops(), 4)
+    out["tasks_per_s"] = round(len(res) / sp, 3)
+    out["span_s"] = round(sp, 4)
+    return out
+
+
+def cmd_c4(a, mx):
+    fd = mx.fn_register(mx.decode_desc(GPT2S))
+    fm = mx.fn_register(mx.mpnn_desc(MPNN, MOLS, MOLS * 30, MOLS * 32))
+    mol_cache = [molecules(k, MOLS) for k in range(1, a.mol_variants + 1)]
+    mfl = float(np.mean([mpnn_task_flops(m, MPNN.hidden, MPNN.steps) for m in mol_cache]))
+    rows = {}
+    for n in [int(x) for x in a.layouts.split(",")]:
+        parts = [mx.part_create(0, s, 1 << 30) for s in LAYOUTS_FILL[n]]
+        for p in parts:
+            mx.fn_load(fd, p)
+            mx.fn_load(fm, p)
+        warm = mixed_items(mx, fd, fm, len(parts), len(parts), mol_cache)
+        closed_batch(mx, [(mx.MX_PART_ANY, t) for _, t in warm])
+        items = mixed_items(mx, fd, fm, a.decode, a.mpnn, mol_cache)
+        res, wall = closed_batch(mx, [(mx.MX_PART_ANY, t) for _, t in items])
+        rows[str(n)] = {"sms": LAYOUTS_FILL[n], **class_stats(res, [k for k, _ in items], mfl,
+                                                              a.decode, a.mpnn),
+                        "e2e_tasks_per_s": round(len(res) / wall, 3)}
+        for p in parts:
+            mx.part_destroy(p)
+    if "1" in rows:
+        for k, v in rows.items():
+            v["ratio_vs_1_partition"] = round(v["tasks_per_s"] / rows["1"]["tasks_per_s"], 3)
+    return {"suite": "D4 c4", "workload": f"configs[3]: {a.decode} GPT-2s decode (B1 P16 G32) + "
+            f"{a.mpnn} MPNN ({MOLS} molecules) tasks shuffled (seed 42), WLAW placement, both "
+            "functions loaded on every partition", "mpnn_flops_per_task": mfl,
+            "peak_gbs": peak_gbs(), "peak_bf16_tflops": peak_bf16_tflops(), "layouts": rows}
+
+
+LAYOUT_B = [40, 40, 16, 16, 16, 8, 8]
+
+
+def apply_layout(mx, parts, sizes):
+    """Resize partitions to `sizes` (shrinks first so growing ones find free groups)."""
+    cur = [mx.part_query(p)["sm_count"] for p in parts]
+    order = sorted(range(len(parts)), key=lambda i: sizes[i] - cur[i])
+    lat_ms = []
+    for i in order:
+        if sizes[i] != cur[i]:
+            h0 = time.perf_counter()
+            mx.part_resize(parts[i], sizes[i], 0)
+            lat_ms.append((time.perf_counter() - h0) * 1e3)
+    return lat_ms
+
+
+def cmd_c5(a, mx):
+    fd = mx.fn_register(mx.decode_desc(GPT2S))
+    fm = mx.fn_register(mx.mpnn_desc(MPNN, MOLS, MOLS * 30, MOLS * 32))
+    mol_cache = [molecules(k, MOLS) for k in range(1, a.mol_variants + 1)]
+    mfl = float(np.mean([mpnn_task_flops(m, MPNN.hidden, MPNN.steps) for m in mol_cache]))
+    out = {"suite": "D5 c5", "workload": f"configs[4]: task farm of {a.tasks} tasks, 50/50 "
+           "GPT-2s decode / MPNN, shuffled (seed 42), WLAW over 7 fill partitions, layout "
+           f"alternating fill-7 <-> {LAYOUT_B} via part_resize after every {a.resize_every} "
+           "submissions", "peak_gbs": peak_gbs()}
+    A = LAYOUTS_FILL[7]
+    for label, sizes, n_tasks in (("partitioned", A, a.tasks), ("1_partition", [148], a.base_tasks)):
+        parts = [mx.part_create(0, s, 1 << 30) for s in sizes]
+        for p in parts:
+            mx.fn_load(fd, p)
+            mx.fn_load(fm, p)
+        warm = mixed_items(mx, fd, fm, len(parts), len(parts), mol_cache)
+        closed_batch(mx, [(mx.MX_PART_ANY, t) for _, t in warm])
+        items = mixed_items(mx, fd, fm, n_tasks // 2, n_tasks - n_tasks // 2, mol_cache)
+        resize_ms = []
+        h0 = time.perf_counter()
+        use_b = False
+        for i, (_, t) in enumerate(items):
+            if label == "partitioned" and i > 0 and i % a.resize_every == 0:
+                use_b = not use_b
+                resize_ms += apply_layout(mx, parts, LAYOUT_B if use_b else A)
+            mx.fn_submit(mx.MX_PART_ANY, t)
+        res = [mx.fn_wait(t) for _, t in items]
+        wall = time.perf_counter() - h0
+        assert all(r["status"] == 0 for r in res)
+        st = class_stats(res, [k for k, _ in items], mfl, n_tasks // 2, n_tasks - n_tasks // 2)
+        st["tasks"] = n_tasks
+        st["e2e_tasks_per_s"] = round(n_tasks / wall, 3)
+        if resize_ms:
+            st["part_resize_ms"] = {"n": len(resize_ms), **{k: round(v, 3) for k, v in
+                                                            percentiles(resize_ms).items()},
+                                    "max": round(max(resize_ms), 3)}
+        out[label] = st
+        for p in parts:
+            mx.part_destroy(p)
+    out["ratio_vs_1_partition"] = round(out["partitioned"]["tasks_per_s"]
+                                        / out["1_partition"]["tasks_per_s"], 3)
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    sub = ap.add_subparsers(dest="cmd", required=True)
+    s = sub.add_parser("smsweep")
+    s.add_argument("--sms", default="4,8,12,16,24,32,48,64,72,96,120,144,148")
+    s.add_argument("--tasks", type=int, default=4)
+    s = sub.add_parser("c3")
+    s.add_argument("--layouts", default="1,2,4")
+    s.add_argument("--batches", default="1,2,4,8")
+    s.add_argument("--tasks", type=int, default=100)
+    s = sub.add_parser("c4")
+    s.add_argument("--layouts", default="1,7")
+    s.add_argument("--decode", type=int, default=700)
+    s.add_argument("--mpnn", type=int, default=700)
+    s.add_argument("--mol-variants", type=int, default=16)
+    s = sub.add_parser("c5")
+    s.add_argument("--tasks", type=int, default=10000)
+    s.add_argument("--base-tasks", type=int, default=1000)
+    s.add_argument("--resize-every", type=int, default=1000)
+    s.add_argument("--mol-variants", type=int, default=16)
+    a = ap.parse_args()
+    from paper_conf_sc_dhakalrwercfm23_b200 import mx
+    mx.mx_init([0])
+    try:
+        out = globals()[f"cmd_{a.cmd}"](a, mx)
+    finally:
+        mx.mx_shutdown()
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()
