@@ -128,7 +128,8 @@ typedef struct {
   int32_t whole;          /* 1 = the whole device (all groups + remainder)            */
   uint64_t group_mask;    /* bit g = 8-SM group g of the device split                  */
   uint64_t hbm_quota, hbm_used, hbm_peak;
-  uint32_t epoch, reserved;
+  uint32_t epoch;
+  uint32_t shared;        /* 1 = unpartitioned stream (part_create_shared, N1)        */
 } mx_part_info;
 
 typedef struct {
@@ -166,6 +167,20 @@ const char* mx_last_error(void);   /* thread-local detail of the last failure   
  * isolation). Errors: MX_ENODEV, MX_EINVAL, MX_ENOSM, MX_ENOMEM (sum of quotas
  * would exceed device memory, I5).                                         */
 mx_status part_create(int32_t gpu, int32_t sm_count, uint64_t hbm_bytes, int32_t* out_part);
+/* Unpartitioned comparison mode (Table 1
+ * and §5.2: time-sharing vs MPS vs MIG). The partition is a plain
+ * stream of the primary context: it owns NO SM groups (not counted in the
+ * 148-SM budget, I2), its kernels may run on any SM, and decode grids are
+ * `n_ctas` CTAs launched cooperatively (all CTAs co-resident or none).
+ *   n_ctas = SM count  -> every task wants the whole GPU: tasks of different
+ *                          shared partitions take turns (time-sharing analog);
+ *   n_ctas = SMs / N   -> N partitions run side by side on hardware-chosen SMs
+ *                          (default-MPS analog, no isolation).
+ * `n_ctas` (clamped to the SM count) is also the partition's WLAW weight. The
+ * HBM quota is enforced as for part_create. part_resize(part, n, 0) changes
+ * the grid size; the partition stays shared. Errors as part_create, except
+ * MX_ENOSM (no groups are taken).                                           */
+mx_status part_create_shared(int32_t gpu, int32_t n_ctas, uint64_t hbm_bytes, int32_t* out_part);
 /* Live re-partition (the paper's future work, §7): new SM group set (own
  * groups released first) -> new green context + stream; queued tasks go to the
  * new stream, in-flight ones finish on the old. Weights never move or reload.
@@ -233,6 +248,8 @@ mx_sched* mx_sched_new(int32_t n_gpus, int32_t n_groups, int32_t group_size, int
                        uint64_t mem_bytes);
 void mx_sched_free(mx_sched* s);
 mx_status mx_sched_create(mx_sched* s, int32_t gpu, int32_t sm_count, uint64_t hbm, int32_t* out_part);
+mx_status mx_sched_create_shared(mx_sched* s, int32_t gpu, int32_t n_ctas, uint64_t hbm,
+                                 int32_t* out_part);
 mx_status mx_sched_resize(mx_sched* s, int32_t part, int32_t sm_count, uint64_t hbm);
 mx_status mx_sched_destroy(mx_sched* s, int32_t part);
 mx_status mx_sched_submit(mx_sched* s, int32_t fn, int32_t part, uint64_t cost,

@@ -30,6 +30,9 @@ def i2_sm_budget(records, total_sms: int = 148) -> list:
     for r in records:
         typ = r[0]
         if typ in (REC_CREATE, REC_RESIZE):
+            if r[7] & 2:            # shared (unpartitioned) stream: owns no SMs
+                live.pop(r[1], None)
+                continue
             live[r[1]] = (r[2], r[3], r[4])
         elif typ == REC_DESTROY:
             live.pop(r[1], None)

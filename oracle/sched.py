@@ -18,7 +18,9 @@ Rules written out (the C++ runtime implements the same rules independently):
     exactly as (A_p + c_k)*s_q < (A_q + c_k)*s_p, ties -> lowest part id;
     then A_p += c_k. A_p is never decremented (timing-independent). Explicit
     placements add c_k to A_p as well.
-  * trace: little-endian records of 8 x u64; timestamps excluded.
+  * trace: little-endian records of 8 x u64; timestamps excluded. CREATE /
+    RESIZE carry a flag word (bit0 whole device, bit1 shared = unpartitioned).
+  * shared partitions (N1) own no groups and do not count toward I2.
 """
 from __future__ import annotations
 
@@ -51,6 +53,7 @@ class Part:
     live: bool = True
     assigned: int = 0
     seq: int = 0
+    shared: bool = False
 
     @property
     def mask(self) -> int:
@@ -113,6 +116,24 @@ class Sim:
         self.records.append((REC_CREATE, p.pid, gpu, smc, p.mask, hbm, 0, int(whole)))
         return p.pid
 
+    def create_shared(self, gpu: int, n_ctas: int, hbm: int) -> int:
+        """Unpartitioned stream on the whole device (the
+        time-sharing / default-MPS comparison modes of PAPER.md Table 1):
+        owns no SM groups, sm_count = min(n_ctas, total_sms) is its grid and WLAW weight."""
+        if gpu < 0 or gpu >= self.n_gpus:
+            raise SchedError(MX_ENODEV)
+        if n_ctas <= 0 or hbm <= 0:
+            raise SchedError(MX_EINVAL)
+        if not self._quota_ok(gpu, hbm):
+            raise SchedError(MX_ENOMEM)
+        p = Part(len(self.parts), gpu, [], min(n_ctas, self.total_sms), False, hbm, shared=True)
+        self.parts.append(p)
+        self.records.append((REC_CREATE, p.pid, gpu, p.sm_count, 0, hbm, 0, 2))
+        return p.pid
+
+    def _flags(self, p: Part) -> int:
+        return int(p.whole) | (2 if p.shared else 0)
+
     def _live(self, pid: int) -> Part:
         if pid < 0 or pid >= len(self.parts) or not self.parts[pid].live:
             raise SchedError(MX_EINVAL)
@@ -124,10 +145,13 @@ class Sim:
         hbm = p.quota if hbm == 0 else hbm
         if not self._quota_ok(p.gpu, hbm, exclude=pid):
             raise SchedError(MX_ENOMEM)
-        groups, smc, whole = self._alloc(p.gpu, sm, exclude=pid)
+        if p.shared:
+            groups, smc, whole = [], min(sm, self.total_sms), False
+        else:
+            groups, smc, whole = self._alloc(p.gpu, sm, exclude=pid)
         p.groups, p.sm_count, p.whole, p.quota = groups, smc, whole, hbm
         p.epoch += 1
-        self.records.append((REC_RESIZE, pid, p.gpu, smc, p.mask, hbm, p.epoch, int(whole)))
+        self.records.append((REC_RESIZE, pid, p.gpu, smc, p.mask, hbm, p.epoch, self._flags(p)))
 
     def destroy(self, pid: int):
         p = self._live(pid)

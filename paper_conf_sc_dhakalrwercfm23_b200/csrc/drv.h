@@ -54,6 +54,7 @@ namespace mx {
   X(cuMemHostGetDevicePointer)     \
   X(cuStreamQuery)                 \
   X(cuLaunchKernel)                \
+  X(cuLaunchCooperativeKernel)     \
   X(cuKernelSetAttribute)          \
   X(cuGetErrorString)
 

@@ -11,7 +11,7 @@ namespace mxk {
 __host__ __device__ inline int round256_h(int k) { return (k + 255) & ~255; }
 
 template <int B>
-int launch_b(const DecodeParams& p, void* stream);
+int launch_b(const DecodeParams& p, void* stream, int cooperative);
 template <int B>
 int set_attrs_b(int device);
 
@@ -34,16 +34,16 @@ uint64_t decode_barriers(int L, int P, int G, int fuse_att) {
   return S * (uint64_t)(fuse_att ? 4 : 5) * (uint64_t)L + (uint64_t)G;   // phases_per_layer() x L + G LM phases
 }
 
-int launch_decode(const DecodeParams& p, void* stream) {
+int launch_decode(const DecodeParams& p, void* stream, int cooperative) {
   switch (p.B) {
-    case 1: return launch_b<1>(p, stream);
-    case 2: return launch_b<2>(p, stream);
-    case 3: return launch_b<3>(p, stream);
-    case 4: return launch_b<4>(p, stream);
-    case 5: return launch_b<5>(p, stream);
-    case 6: return launch_b<6>(p, stream);
-    case 7: return launch_b<7>(p, stream);
-    case 8: return launch_b<8>(p, stream);
+    case 1: return launch_b<1>(p, stream, cooperative);
+    case 2: return launch_b<2>(p, stream, cooperative);
+    case 3: return launch_b<3>(p, stream, cooperative);
+    case 4: return launch_b<4>(p, stream, cooperative);
+    case 5: return launch_b<5>(p, stream, cooperative);
+    case 6: return launch_b<6>(p, stream, cooperative);
+    case 7: return launch_b<7>(p, stream, cooperative);
+    case 8: return launch_b<8>(p, stream, cooperative);
     default: return -4;
   }
 }

@@ -934,7 +934,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
 }
 
 template <int B>
-int launch_b(const DecodeParams& p, void* stream) {
+int launch_b(const DecodeParams& p, void* stream, int cooperative) {
   const int kmax = max(max(p.d, p.q_dim), p.ff);
   int ns = 0;
   const int smem = decode_smem_bytes(B, kmax, &ns);
@@ -943,7 +943,7 @@ int launch_b(const DecodeParams& p, void* stream) {
   int ns_arg = ns, kmax_arg = kmax;
   void* args[] = {&pc, &ns_arg, &kmax_arg};
   return launch_kernel(decode_kernel<B>, dim3(p.n_ctas), dim3(kDecodeThreads), (unsigned)smem,
-                       stream, args);
+                       stream, args, cooperative != 0);
 }
 
 template <int B>
@@ -956,6 +956,6 @@ int set_attrs_b(int device) {
 // One translation unit per batch size (parallel compilation).
 #define MX_DECODE_INSTANTIATE(B)                                      \
   namespace mxk {                                                     \
-  template int launch_b<B>(const DecodeParams& p, void* stream);      \
+  template int launch_b<B>(const DecodeParams& p, void* stream, int); \
   template int set_attrs_b<B>(int device);                            \
   }

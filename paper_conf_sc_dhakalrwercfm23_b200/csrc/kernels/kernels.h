@@ -74,7 +74,9 @@ uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 // Shared-memory bytes of the decode kernel for a given shape.
 int decode_smem_bytes(int B, int kmax, int* n_stages);
 
-int launch_decode(const DecodeParams& p, void* stream);
+// cooperative != 0: cuLaunchCooperativeKernel (all CTAs co-resident; used on
+// unpartitioned streams where other kernels compete for the same SMs).
+int launch_decode(const DecodeParams& p, void* stream, int cooperative = 0);
 int launch_fill_weights(uint16_t* dst, uint64_t n, uint64_t seed, uint32_t tid, int is_gain,
                         int n_ctas, void* stream);
 int launch_rope_table(float* dst, int max_seq, int hd, float theta, void* stream);

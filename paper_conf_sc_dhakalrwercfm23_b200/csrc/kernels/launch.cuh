@@ -15,6 +15,8 @@ namespace mxk {
 struct DriverLaunch {
   CUresult (*launch)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                      unsigned, CUstream, void**, void**) = nullptr;
+  CUresult (*launch_coop)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                          unsigned, CUstream, void**) = nullptr;
   CUresult (*kernel_set_attr)(CUfunction_attribute, int, CUkernel, CUdevice) = nullptr;
 };
 
@@ -22,13 +24,18 @@ DriverLaunch& driver_launch();
 std::atomic<uint64_t>& launch_count_ref();
 
 template <typename K>
-inline int launch_kernel(K* kern, dim3 grid, dim3 block, unsigned smem, void* stream, void** args) {
+inline int launch_kernel(K* kern, dim3 grid, dim3 block, unsigned smem, void* stream, void** args,
+                         bool cooperative = false) {
   cudaKernel_t k = nullptr;
   if (cudaGetKernel(&k, reinterpret_cast<const void*>(kern)) != cudaSuccess || !k) return -1;
   DriverLaunch& d = driver_launch();
-  if (!d.launch) return -2;
-  CUresult r = d.launch(reinterpret_cast<CUfunction>(k), grid.x, grid.y, grid.z, block.x, block.y,
-                        block.z, smem, reinterpret_cast<CUstream>(stream), args, nullptr);
+  if (!d.launch || (cooperative && !d.launch_coop)) return -2;
+  CUresult r = cooperative
+                   ? d.launch_coop(reinterpret_cast<CUfunction>(k), grid.x, grid.y, grid.z, block.x,
+                                   block.y, block.z, smem, reinterpret_cast<CUstream>(stream), args)
+                   : d.launch(reinterpret_cast<CUfunction>(k), grid.x, grid.y, grid.z, block.x,
+                              block.y, block.z, smem, reinterpret_cast<CUstream>(stream), args,
+                              nullptr);
   if (r != CUDA_SUCCESS) return (int)r;
   launch_count_ref().fetch_add(1, std::memory_order_relaxed);
   return 0;

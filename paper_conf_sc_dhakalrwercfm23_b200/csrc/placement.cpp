@@ -6,6 +6,8 @@
 //  * ANY: weighted least-assigned-work, argmin (A_p + c)/s_p compared exactly
 //    in 128-bit integers, ties -> lowest part id; A_p += c for every placement.
 //  * STATIC equal division (A6) is done by the caller with explicit parts.
+//  * shared partitions (N1, unpartitioned comparison modes) own no groups; their
+//    sm_count is the grid size (<= total_sms); record flag word: bit0 whole, bit1 shared.
 #include "placement.h"
 
 #include "../../include/mx.h"
@@ -81,7 +83,30 @@ int Sched::create(int gpu, int sm, uint64_t hbm, int* out_part) {
   p.live = true;
   parts_.push_back(p);
   int id = (int)parts_.size() - 1;
-  record(REC_CREATE, (uint64_t)id, (uint64_t)gpu, (uint64_t)smc, p.mask(), hbm, 0, whole ? 1 : 0);
+  record(REC_CREATE, (uint64_t)id, (uint64_t)gpu, (uint64_t)smc, p.mask(), hbm, 0, flags(p));
+  *out_part = id;
+  return MX_OK;
+}
+
+int Sched::plan_create_shared(int gpu, int n_ctas, uint64_t hbm) const {
+  if (gpu < 0 || gpu >= n_gpus_) return MX_ENODEV;
+  if (n_ctas <= 0 || hbm == 0) return MX_EINVAL;
+  if (!quota_ok(gpu, hbm, -1)) return MX_ENOMEM;
+  return MX_OK;
+}
+
+int Sched::create_shared(int gpu, int n_ctas, uint64_t hbm, int* out_part) {
+  int rc = plan_create_shared(gpu, n_ctas, hbm);
+  if (rc) return rc;
+  SchedPart p;
+  p.gpu = gpu;
+  p.sm_count = n_ctas < total_sms_ ? n_ctas : total_sms_;
+  p.shared = true;
+  p.quota = hbm;
+  p.live = true;
+  parts_.push_back(p);
+  int id = (int)parts_.size() - 1;
+  record(REC_CREATE, (uint64_t)id, (uint64_t)gpu, (uint64_t)p.sm_count, 0, hbm, 0, flags(p));
   *out_part = id;
   return MX_OK;
 }
@@ -94,6 +119,12 @@ int Sched::plan_resize(int part, int sm, uint64_t hbm, std::vector<int>* groups,
   if (hbm == 0) hbm = p.quota;
   if (!quota_ok(p.gpu, hbm, part)) return MX_ENOMEM;
   *quota = hbm;
+  if (p.shared) {   // stays unpartitioned: only the grid size changes
+    groups->clear();
+    *smc = sm < total_sms_ ? sm : total_sms_;
+    *whole = false;
+    return MX_OK;
+  }
   return alloc(p.gpu, sm, part, groups, smc, whole);
 }
 
@@ -111,7 +142,7 @@ int Sched::resize(int part, int sm, uint64_t hbm) {
   p.quota = quota;
   p.epoch += 1;
   record(REC_RESIZE, (uint64_t)part, (uint64_t)p.gpu, (uint64_t)smc, p.mask(), quota, p.epoch,
-         whole ? 1 : 0);
+         flags(p));
   return MX_OK;
 }
 

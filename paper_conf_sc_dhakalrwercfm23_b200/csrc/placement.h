@@ -19,6 +19,7 @@ struct SchedPart {
   std::vector<int> groups;   // ascending group indices
   int32_t sm_count = 0;
   bool whole = false;
+  bool shared = false;       // N1: no SM groups; runs anywhere on the device (sm_count = grid)
   uint64_t quota = 0;
   uint32_t epoch = 0;
   bool live = false;
@@ -43,6 +44,10 @@ class Sched {
   Sched(int n_gpus, int n_groups, int group_size, int total_sms, uint64_t mem_bytes);
   // All return an mx_status code (0 ok).
   int create(int gpu, int sm, uint64_t hbm, int* out_part);
+  // Unpartitioned ("shared") partition: a stream on the whole device that owns
+  // no SM groups (not counted in I2); n_ctas is its grid size and its WLAW weight.
+  int create_shared(int gpu, int n_ctas, uint64_t hbm, int* out_part);
+  int plan_create_shared(int gpu, int n_ctas, uint64_t hbm) const;
   int resize(int part, int sm, uint64_t hbm);
   int destroy(int part);
   int submit(int fn, int part, uint64_t cost, Placement* out);
@@ -58,6 +63,7 @@ class Sched {
  private:
   int alloc(int gpu, int sm, int exclude, std::vector<int>* groups, int* smc, bool* whole) const;
   bool quota_ok(int gpu, uint64_t quota, int exclude) const;
+  uint64_t flags(const SchedPart& p) const { return (p.whole ? 1u : 0u) | (p.shared ? 2u : 0u); }
   void record(uint64_t a, uint64_t b, uint64_t c, uint64_t d, uint64_t e, uint64_t f, uint64_t g, uint64_t h);
 
   int n_gpus_, n_groups_, group_size_, total_sms_;

@@ -262,6 +262,25 @@ static void destroy_exec(Exec* e) {
   if (e->gctx) drv().cuGreenCtxDestroy(e->gctx);
 }
 
+// Unpartitioned exec (N1): a non-blocking stream of the primary context.
+static int make_shared_exec(Gpu& gpu, int n_ctas, uint32_t epoch, std::unique_ptr<Exec>* out) {
+  auto e = std::make_unique<Exec>();
+  e->epoch = epoch;
+  e->shared = true;
+  e->ctx = gpu.primary;
+  e->n_ctas = n_ctas < gpu.sm_total ? n_ctas : gpu.sm_total;
+  CtxGuard g(gpu.primary);
+  CU_TRY(drv().cuStreamCreate(&e->stream, CU_STREAM_NON_BLOCKING));
+  for (auto& lane : e->ev)
+    for (auto& ev : lane)
+      if (drv().cuEventCreate(&ev, CU_EVENT_DEFAULT) != CUDA_SUCCESS) {
+        set_error("cuEventCreate failed");
+        return MX_EDEVICE;
+      }
+  *out = std::move(e);
+  return MX_OK;
+}
+
 static int make_exec(Gpu& gpu, const std::vector<int>& groups, bool whole, uint32_t epoch,
                      std::unique_ptr<Exec>* out) {
   auto e = std::make_unique<Exec>();
@@ -616,7 +635,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.err = reinterpret_cast<int*>(s.err);
     k.prof = g_decode_prof ? reinterpret_cast<unsigned long long*>(p.sys + 65536) : nullptr;
     if (!t->use_flag) CU_TRY(drv().cuEventRecord(ev[0], st));
-    int rc = mxk::launch_decode(k, st);
+    int rc = mxk::launch_decode(k, st, e->shared ? 1 : 0);
     if (rc) {
       set_error("decode launch failed (%d)", rc);
       return MX_EDEVICE;
@@ -932,6 +951,7 @@ static int init_impl(const std::vector<int>& ordinals) {
     return MX_ENODEV;
   }
   mxk::driver_launch().launch = drv().cuLaunchKernel;
+  mxk::driver_launch().launch_coop = drv().cuLaunchCooperativeKernel;
   mxk::driver_launch().kernel_set_attr = drv().cuKernelSetAttribute;
   if (drv().cuInit(0) != CUDA_SUCCESS) {
     set_error("cuInit failed: no usable GPU");
@@ -1135,6 +1155,43 @@ mx_status part_create(int32_t gpu, int32_t sm_count, uint64_t hbm_bytes, int32_t
   return MX_OK;
 }
 
+mx_status part_create_shared(int32_t gpu, int32_t n_ctas, uint64_t hbm_bytes, int32_t* out_part) {
+  MX_REQUIRE_INIT();
+  if (!out_part) return MX_EINVAL;
+  std::lock_guard<std::mutex> lk(L->mu);
+  int rc = L->sched->plan_create_shared(gpu, n_ctas, hbm_bytes);
+  if (rc) {
+    set_error("part_create_shared(gpu=%d, n_ctas=%d, hbm=%llu): %s", gpu, n_ctas,
+              (unsigned long long)hbm_bytes, mx_strerror(rc));
+    return rc;
+  }
+  Gpu& g = *L->gpus[gpu];
+  CtxGuard cg(g.primary);
+  auto p = std::make_unique<Partition>();
+  p->gpu = gpu;
+  rc = make_shared_exec(g, n_ctas, 0, &p->cur);
+  if (rc) return rc;
+  rc = p->arena.init(g.ordinal, hbm_bytes, g.mem_bytes);
+  if (rc == MX_OK) rc = p->arena.alloc(128 * 1024, 256, &p->sys);
+  int id = -1;
+  if (rc == MX_OK) rc = L->sched->create_shared(gpu, n_ctas, hbm_bytes, &id);
+  if (rc || id != (int)L->parts.size()) {
+    destroy_exec(p->cur.get());
+    p->arena.release();
+    set_error("part_create_shared: arena or scheduler failure");
+    return rc ? rc : MX_EDEVICE;
+  }
+  p->id = id;
+  Partition* raw = p.get();
+  L->parts.push_back(std::move(p));
+  {
+    std::lock_guard<std::mutex> glk(g.mu);
+    g.parts.push_back(raw);
+  }
+  *out_part = id;
+  return MX_OK;
+}
+
 mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
   MX_REQUIRE_INIT();
   std::lock_guard<std::mutex> lk(L->mu);
@@ -1160,7 +1217,7 @@ mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
   }
   CtxGuard cg(g.primary);
   const SchedPart& sp = L->sched->part(part);
-  const bool same_sms = (groups == sp.groups && whole == sp.whole);
+  const bool same_sms = sp.shared || (groups == sp.groups && whole == sp.whole);
   std::unique_ptr<Exec> ne;
   if (!same_sms) {
     rc = make_exec(g, groups, whole, sp.epoch + 1, &ne);
@@ -1184,6 +1241,7 @@ mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
       p.cur = std::move(ne);
     } else {
       p.cur->epoch = sp.epoch + 1;
+      if (sp.shared) p.cur->n_ctas = smc;   // unpartitioned: only the grid size changes
     }
     p.arena.set_quota(quota);
   }
@@ -1240,7 +1298,7 @@ mx_status part_query(int32_t part, mx_part_info* out) {
   out->hbm_used = p.arena.used();
   out->hbm_peak = p.arena.peak();
   out->epoch = sp.epoch;
-  out->reserved = 0;
+  out->shared = sp.shared ? 1u : 0u;
   return MX_OK;
 }
 
@@ -1544,6 +1602,12 @@ void mx_sched_free(mx_sched* s) { delete s; }
 mx_status mx_sched_create(mx_sched* s, int32_t gpu, int32_t sm_count, uint64_t hbm, int32_t* out_part) {
   if (!s || !out_part) return MX_EINVAL;
   return s->s.create(gpu, sm_count, hbm, out_part);
+}
+
+mx_status mx_sched_create_shared(mx_sched* s, int32_t gpu, int32_t n_ctas, uint64_t hbm,
+                                 int32_t* out_part) {
+  if (!s || !out_part) return MX_EINVAL;
+  return s->s.create_shared(gpu, n_ctas, hbm, out_part);
 }
 
 mx_status mx_sched_resize(mx_sched* s, int32_t part, int32_t sm_count, uint64_t hbm) {

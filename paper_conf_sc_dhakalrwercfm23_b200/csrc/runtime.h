@@ -36,6 +36,7 @@ struct Exec {
   CUcontext ctx = nullptr;
   CUstream stream = nullptr;
   int n_ctas = 0;          // SMs provisioned (persistent grid size)
+  bool shared = false;     // primary-context stream, no SM restriction (N1); cooperative launches
   uint32_t epoch = 0;
   CUevent ev[2][3] = {};   // per in-flight lane: kernel start, kernel end, done
   int inflight = 0;

@@ -65,7 +65,7 @@ class PartInfoC(C.Structure):
     _fields_ = [("gpu", C.c_int32), ("sm_count", C.c_int32), ("n_ctas", C.c_int32),
                 ("whole", C.c_int32), ("group_mask", C.c_uint64), ("hbm_quota", C.c_uint64),
                 ("hbm_used", C.c_uint64), ("hbm_peak", C.c_uint64), ("epoch", C.c_uint32),
-                ("reserved", C.c_uint32)]
+                ("shared", C.c_uint32)]
 
 
 class GpuInfoC(C.Structure):
@@ -84,6 +84,7 @@ _SIGS = {
     "mx_strerror": (C.c_char_p, [C.c_int32]),
     "mx_last_error": (C.c_char_p, []),
     "part_create": (C.c_int32, [C.c_int32, C.c_int32, C.c_uint64, C.POINTER(C.c_int32)]),
+    "part_create_shared": (C.c_int32, [C.c_int32, C.c_int32, C.c_uint64, C.POINTER(C.c_int32)]),
     "part_resize": (C.c_int32, [C.c_int32, C.c_int32, C.c_uint64]),
     "part_destroy": (C.c_int32, [C.c_int32]),
     "part_query": (C.c_int32, [C.c_int32, C.POINTER(PartInfoC)]),
@@ -104,6 +105,8 @@ _SIGS = {
     "mx_sched_free": (None, [C.c_void_p]),
     "mx_sched_create": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64,
                                     C.POINTER(C.c_int32)]),
+    "mx_sched_create_shared": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64,
+                                           C.POINTER(C.c_int32)]),
     "mx_sched_resize": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64]),
     "mx_sched_destroy": (C.c_int32, [C.c_void_p, C.c_int32]),
     "mx_sched_submit": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64,
@@ -179,6 +182,13 @@ def mx_gpu_query(gpu: int) -> dict:
 def part_create(gpu: int, sm_count: int, hbm_bytes: int) -> int:
     p = C.c_int32()
     _check(lib().part_create(gpu, sm_count, hbm_bytes, C.byref(p)), "part_create")
+    return p.value
+
+
+def part_create_shared(gpu: int, n_ctas: int, hbm_bytes: int) -> int:
+    """Unpartitioned stream (N1 comparison modes): no SM groups, grid = n_ctas."""
+    p = C.c_int32()
+    _check(lib().part_create_shared(gpu, n_ctas, hbm_bytes, C.byref(p)), "part_create_shared")
     return p.value
 
 
@@ -354,6 +364,12 @@ class HostSched:
     def create(self, gpu, sm, hbm) -> int:
         p = C.c_int32()
         _check(lib().mx_sched_create(self.h, gpu, sm, hbm, C.byref(p)), "mx_sched_create")
+        return p.value
+
+    def create_shared(self, gpu, n_ctas, hbm) -> int:
+        p = C.c_int32()
+        _check(lib().mx_sched_create_shared(self.h, gpu, n_ctas, hbm, C.byref(p)),
+               "mx_sched_create_shared")
         return p.value
 
     def resize(self, part, sm, hbm):

@@ -49,6 +49,8 @@ def _replay(events, n_gpus=2):
         try:
             if kind == "c":
                 sim.create(a % n_gpus, b, c)
+            elif kind == "x":
+                sim.create_shared(a % n_gpus, b, c)
             elif kind == "r":
                 sim.resize(a % max(1, len(sim.parts)), b, c)
             elif kind == "d":
@@ -60,6 +62,8 @@ def _replay(events, n_gpus=2):
         try:
             if kind == "c":
                 cpp.create(a % n_gpus, b, c)
+            elif kind == "x":
+                cpp.create_shared(a % n_gpus, b, c)
             elif kind == "r":
                 cpp.resize(a % max(1, len(sim.parts)), b, c)
             elif kind == "d":
@@ -75,13 +79,14 @@ def _replay(events, n_gpus=2):
 def test_cpp_placement_trace_equals_simulator_fixed():
     ev = [("c", 0, 72, 100), ("c", 0, 72, 100), ("c", 1, 16, 10), ("s", 0, 1, 500),
           ("s", 1, 2, 700), ("r", 0, 40, 0), ("s", 2, 1, 50), ("d", 2, 0, 0), ("s", 3, 1, 9),
-          ("c", 1, 148, 10), ("c", 1, 8, 10), ("c", 0, 20, 999)]
+          ("c", 1, 148, 10), ("c", 1, 8, 10), ("c", 0, 20, 999), ("x", 0, 37, 10),
+          ("x", 0, 500, 10), ("s", 1, 1, 77), ("r", 4, 74, 0), ("x", 1, 0, 5)]
     sim, cpp = _replay(ev)
     assert cpp.trace_bytes() == sim.trace_bytes()
 
 
 @settings(max_examples=200, deadline=None)
-@given(st.lists(st.tuples(st.sampled_from("crds"), st.integers(0, 20), st.integers(-5, 160),
+@given(st.lists(st.tuples(st.sampled_from("crdsx"), st.integers(0, 20), st.integers(-5, 160),
                           st.integers(0, 400)), max_size=50))
 def test_cpp_placement_trace_equals_simulator_random(events):
     sim, cpp = _replay(events)

@@ -106,7 +106,7 @@ def test_trace_format_roundtrip():
     assert len(sim.trace_sha256()) == 64
 
 
-events = st.lists(st.tuples(st.sampled_from(["c", "r", "d", "s"]), st.integers(0, 2),
+events = st.lists(st.tuples(st.sampled_from(["c", "r", "d", "s", "x"]), st.integers(0, 2),
                             st.integers(1, 160), st.integers(1, 40)), min_size=1, max_size=60)
 
 
@@ -118,6 +118,8 @@ def test_random_event_streams_keep_invariants(evs):
         try:
             if kind == "c":
                 sim.create(gpu, sm, x)
+            elif kind == "x":
+                sim.create_shared(gpu, sm, x)
             elif kind == "r" and sim.parts:
                 sim.resize(x % len(sim.parts), sm, x)
             elif kind == "d" and sim.parts:
@@ -134,6 +136,31 @@ def test_random_event_streams_keep_invariants(evs):
         if r[0] == S.REC_PLACE:
             assert seqs.get(r[4], -1) + 1 == r[5]       # FIFO seq per partition
             seqs[r[4]] = r[5]
+
+
+def test_shared_partitions_take_no_groups_and_weigh_by_grid():
+    """N1 (Table 1): unpartitioned streams own
+    no SM groups, so the whole device can still be partitioned next to them; their
+    WLAW weight is the grid size: with grids 148 and 37 (4:1) and equal costs,
+    the first 5 ANY placements go 4 to the big grid and 1 to the small one."""
+    sim = S.Sim(1, n_groups=37, group_size=4)
+    a = sim.create_shared(0, 148, 10)
+    b = sim.create_shared(0, 37, 10)
+    assert sim.parts[a].sm_count == 148 and sim.parts[a].groups == []
+    assert sim.create_shared(0, 1000, 10) == 2 and sim.parts[2].sm_count == 148
+    whole = sim.create(0, 148, 10)            # every group is still free
+    assert sim.parts[whole].whole
+    sim.destroy(whole)
+    sim.destroy(2)
+    got = [sim.submit(1, S.MX_PART_ANY, 100)[1] for _ in range(5)]
+    assert sorted(got) == [a, a, a, a, b]
+    sim.resize(b, 74, 0)                      # stays shared, grid 74
+    assert sim.parts[b].groups == [] and sim.parts[b].sm_count == 74
+    recs = S.parse_trace(sim.trace_bytes())
+    assert [r[7] for r in recs if r[0] == S.REC_CREATE] == [2, 2, 2, 1]
+    assert I.i2_sm_budget(recs) == []
+    with pytest.raises(S.SchedError):
+        sim.create_shared(0, 0, 10)
 
 
 def test_invariant_checkers_detect_violations():

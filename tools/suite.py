@@ -296,6 +296,47 @@ def cmd_c5(a, mx):
     return out
 
 
+# ---------------------------------------------------------------------------
+# N1: partitioned (green contexts) vs unpartitioned-concurrent vs time-shared
+# ---------------------------------------------------------------------------
+
+def cmd_modes(a, mx):
+    """PAPER.md Table 1 and Figs. 4-5 compare time-
+    sharing, MPS and MIG. Here, for N concurrent function instances:
+      partitioned  : N green-context partitions (fill layout, SM-isolated)
+      concurrent   : N shared streams, grid = 148/N CTAs each, hardware-placed
+                     (default-MPS analog: concurrent, no isolation)
+      timeshared   : N shared streams, grid = 148 CTAs each (every task wants
+                     the whole GPU, so tasks take turns: time-slicing analog)
+    Same closed batch of GPT-2s decode tasks, STATIC (k-1) mod N placement."""
+    cfg = GPT2S
+    fn = mx.fn_register(mx.decode_desc(cfg))
+    tb = decode_task_bytes(cfg, 1, P_LEN, G_LEN)
+    rows = []
+    for n in [int(x) for x in a.ns.split(",")]:
+        for mode in ("partitioned", "concurrent", "timeshared"):
+            if mode == "partitioned":
+                parts = [mx.part_create(0, s, 512 << 20) for s in LAYOUTS_FILL[n]]
+            else:
+                grid = 148 if mode == "timeshared" else max(1, 148 // n)
+                parts = [mx.part_create_shared(0, grid, 512 << 20) for _ in range(n)]
+            for p in parts:
+                mx.fn_load(fn, p)
+            closed_batch(mx, [(p, mx.decode_task(fn, prompt_tokens(1, 1, P_LEN, cfg.vocab), G_LEN))
+                              for p in parts])
+            items = [(parts[(k - 1) % n], mx.decode_task(fn, prompt_tokens(k, 1, P_LEN, cfg.vocab),
+                                                         G_LEN)) for k in range(1, a.tasks + 1)]
+            res, _ = closed_batch(mx, items)
+            sp = span_s(res)
+            rows.append({"n": n, "mode": mode, "grid": mx.part_query(parts[0])["n_ctas"],
+                         "tasks_per_s": round(a.tasks / sp, 3),
+                         "hbm_frac": round(a.tasks * tb / sp / 1e9 / peak_gbs(), 4), **lat(res)})
+            for p in parts:
+                mx.part_destroy(p)
+    return {"suite": "N1 modes", "workload": f"configs[1] GPT-2s decode B1 P16 G32, {a.tasks} "
+            "tasks per point, STATIC placement", "peak_gbs": peak_gbs(), "rows": rows}
+
+
 def main():
     ap = argparse.ArgumentParser()
     sub = ap.add_subparsers(dest="cmd", required=True)
@@ -316,6 +357,9 @@ def main():
     s.add_argument("--base-tasks", type=int, default=1000)
     s.add_argument("--resize-every", type=int, default=1000)
     s.add_argument("--mol-variants", type=int, default=16)
+    s = sub.add_parser("modes")
+    s.add_argument("--ns", default="1,2,4,7,14")
+    s.add_argument("--tasks", type=int, default=140)
     a = ap.parse_args()
     from paper_conf_sc_dhakalrwercfm23_b200 import mx
     mx.mx_init([0])
