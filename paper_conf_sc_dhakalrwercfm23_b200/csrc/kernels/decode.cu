@@ -8,16 +8,14 @@
 namespace mxk {
 
 
-__host__ __device__ inline int round256_h(int k) { return (k + 255) & ~255; }
-
 template <int B>
 int launch_b(const DecodeParams& p, void* stream, int cooperative);
 template <int B>
 int set_attrs_b(int device);
 
 int decode_smem_bytes(int B, int kmax, int* n_stages) {
-  const int fixed = B * round256_h(kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 + 8 * 4 +
-                    kConsumerWarps * 8 * 4 + 128;
+  const int fixed = B * decode_xin_cols(B, kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 +
+                    8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 128;
   const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;

@@ -51,30 +51,53 @@ constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
 #endif
 constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
 
+// One GEMV phase, or one K segment of it. Phases whose staged activations
+// (B * K * 4 bytes) exceed kXinSegBytes run as `nseg` column segments
+// [k0, k0 + K) inside the owning CTA (split-K): each segment streams the same
+// rows restricted to its columns, partial sums of all but the last segment go
+// to the slot's kacc buffer, and the last segment applies the epilogue to
+// (kacc + partial). Segment widths depend only on the shape, so results stay
+// independent of the partition size.
 struct Phase {
   int kind, layer, R, K, KP, NC, NG, TR;
+  int ldw;         // row stride of the weight matrix in HBM (= the full K)
+  int k0, seg, nseg;
   const uint16_t* w0;
   const uint16_t* w1;
 };
 
 __host__ __device__ __forceinline__ int round256(int k) { return (k + 255) & ~255; }
 
-__device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int layer) {
+template <int B>
+__device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int layer, int seg) {
   Phase ph;
   ph.kind = kind;
   ph.layer = layer;
   ph.w1 = nullptr;
   ph.w0 = nullptr;
   ph.R = 0;
-  ph.K = 0;
+  int K = 0;
   const uint16_t* lw = p.w_layers + (uint64_t)layer * p.layer_stride;
   switch (kind) {
-    case PH_QKV: ph.R = p.qkv_rows; ph.K = p.d; ph.w0 = lw + p.off_wqkv; break;
-    case PH_O: ph.R = p.d; ph.K = p.q_dim; ph.w0 = lw + p.off_wo; break;
-    case PH_GU: ph.R = p.ff; ph.K = p.d; ph.w0 = lw + p.off_wgate; ph.w1 = lw + p.off_wup; break;
-    case PH_DOWN: ph.R = p.d; ph.K = p.ff; ph.w0 = lw + p.off_wdown; break;
-    case PH_LM: ph.R = p.V; ph.K = p.d; ph.w0 = p.lm_head; break;
+    case PH_QKV: ph.R = p.qkv_rows; K = p.d; ph.w0 = lw + p.off_wqkv; break;
+    case PH_O: ph.R = p.d; K = p.q_dim; ph.w0 = lw + p.off_wo; break;
+    case PH_GU: ph.R = p.ff; K = p.d; ph.w0 = lw + p.off_wgate; ph.w1 = lw + p.off_wup; break;
+    case PH_DOWN: ph.R = p.d; K = p.ff; ph.w0 = lw + p.off_wdown; break;
+    case PH_LM: ph.R = p.V; K = p.d; ph.w0 = p.lm_head; break;
     default: break;
+  }
+  ph.ldw = K;
+  constexpr int KS = decode_seg_cols(B);
+  ph.nseg = (K + KS - 1) / KS;
+  if (ph.nseg < 1) ph.nseg = 1;
+  ph.seg = seg;
+  if (ph.nseg > 1) {
+    const int w = round256((K + ph.nseg - 1) / ph.nseg);
+    ph.k0 = seg * w;
+    ph.K = min(w, K - ph.k0);
+  } else {
+    ph.k0 = 0;
+    ph.K = K;
   }
   ph.KP = round256(ph.K);
   ph.NC = ph.KP / 256;
@@ -88,6 +111,13 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
   }
   ph.TR = tr;
   return ph;
+}
+
+template <int B>
+__device__ __forceinline__ int phase_segments(const DecodeParams& p, int kind) {
+  const int K = (kind == PH_O) ? p.q_dim : (kind == PH_DOWN) ? p.ff : p.d;
+  constexpr int KS = decode_seg_cols(B);
+  return kind == PH_ATT ? 1 : max(1, (K + KS - 1) / KS);
 }
 
 // Rows [r0, r1) of a phase owned by this CTA; `rot` rotates the assignment so
@@ -126,15 +156,17 @@ struct Smem {
   unsigned long long* best;  // [8]
   int* tok;                  // [8]
   float* wsum;               // [kConsumerWarps][8]
+  float* inv;                // [8] RMSNorm scale of the phase input (kept across K segments)
 };
 
-__device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int B, int kmax) {
+template <int B>
+__device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int kmax) {
   Smem s;
   uint8_t* p = base;
   s.ring = p;
   p += (size_t)n_stages * kStageBytes;
   s.xin = reinterpret_cast<float*>(p);
-  p += (size_t)B * round256(kmax) * 4;
+  p += (size_t)B * decode_xin_cols(B, kmax) * 4;
   s.red = reinterpret_cast<float*>(p);
   p += (size_t)n_stages * kMaxUnits * B * 4;
   s.cnt = reinterpret_cast<int*>(p);
@@ -150,6 +182,8 @@ __device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int B, int km
   s.tok = reinterpret_cast<int*>(p);
   p += 8 * 4;
   s.wsum = reinterpret_cast<float*>(p);
+  p += (size_t)kConsumerWarps * 8 * 4;
+  s.inv = reinterpret_cast<float*>(p);
   return s;
 }
 
@@ -185,7 +219,8 @@ __device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned lon
 // ---------------------------------------------------------------------------
 // Producer: stream this CTA's weight rows of every phase of every step.
 // ---------------------------------------------------------------------------
-static __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stages) {
+template <int B>
+__device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stages) {
   const int C = p.n_ctas, cta = blockIdx.x, L = p.L;
   const int S = p.P + p.G - 1;
   const int pl = phases_per_layer(p.fuse_att);
@@ -197,7 +232,6 @@ static __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int 
     for (int k = 0; k < nph; ++k) {
       const int kind = phase_kind(k, L, p.fuse_att);
       if (kind == PH_ATT) continue;
-      const Phase ph = make_phase(p, kind, k / pl);
       // L2 prefetch of the small operands the consumers will need a few us from
       // now (they are evicted by the weight stream between steps): the norm
       // gain of this phase, and for QKV(l) the cached keys/values of layer l
@@ -220,26 +254,42 @@ static __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int 
           }
         }
       }
-      int r0, r1;
-      my_rows(ph.R, C, cta, k, &r0, &r1);
-      for (int r = r0; r < r1; r += ph.TR) {
-        const int n = min(ph.TR, r1 - r);
-        // never abandons the stream: after a barrier timeout the consumers run
-        // through the remaining phases without waiting, so every slot is freed.
-        const long long tw = clock64();
-        while (!MX_EMPTY_WAIT(&sm.empty[stage], phase_bit ^ 1u)) {
-        }
-        wait_cyc += clock64() - tw;
-        const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
-        const uint32_t total = (kind == PH_GU) ? 2u * one : one;
-        uint8_t* dst = sm.ring + (size_t)stage * kStageBytes;
-        mbar_arrive_expect_tx(&sm.full[stage], total);
-        bulk_g2s_evict_first(dst, ph.w0 + (size_t)r * ph.K, one, &sm.full[stage], pol);
-        if (kind == PH_GU)
-          bulk_g2s_evict_first(dst + one, ph.w1 + (size_t)r * ph.K, one, &sm.full[stage], pol);
-        if (++stage == (uint32_t)n_stages) {
-          stage = 0;
-          phase_bit ^= 1u;
+      const int nseg = phase_segments<B>(p, kind);
+      for (int seg = 0; seg < nseg; ++seg) {
+        const Phase ph = make_phase<B>(p, kind, k / pl, seg);
+        int r0, r1;
+        my_rows(ph.R, C, cta, k, &r0, &r1);
+        for (int r = r0; r < r1; r += ph.TR) {
+          const int n = min(ph.TR, r1 - r);
+          // never abandons the stream: after a barrier timeout the consumers run
+          // through the remaining phases without waiting, so every slot is freed.
+          const long long tw = clock64();
+          while (!MX_EMPTY_WAIT(&sm.empty[stage], phase_bit ^ 1u)) {
+          }
+          wait_cyc += clock64() - tw;
+          const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
+          const uint32_t total = (kind == PH_GU) ? 2u * one : one;
+          uint8_t* dst = sm.ring + (size_t)stage * kStageBytes;
+          mbar_arrive_expect_tx(&sm.full[stage], total);
+          if (ph.nseg == 1) {
+            // whole rows: one contiguous copy per matrix
+            bulk_g2s_evict_first(dst, ph.w0 + (size_t)r * ph.K, one, &sm.full[stage], pol);
+            if (kind == PH_GU)
+              bulk_g2s_evict_first(dst + one, ph.w1 + (size_t)r * ph.K, one, &sm.full[stage], pol);
+          } else {
+            // K segment: one copy per row of columns [k0, k0 + K), packed
+            const uint32_t rb = (uint32_t)ph.K * 2u;
+            for (int i = 0; i < n; ++i) {
+              const size_t src = (size_t)(r + i) * ph.ldw + ph.k0;
+              bulk_g2s_evict_first(dst + i * rb, ph.w0 + src, rb, &sm.full[stage], pol);
+              if (kind == PH_GU)
+                bulk_g2s_evict_first(dst + one + i * rb, ph.w1 + src, rb, &sm.full[stage], pol);
+            }
+          }
+          if (++stage == (uint32_t)n_stages) {
+            stage = 0;
+            phase_bit ^= 1u;
+          }
         }
       }
     }
@@ -430,11 +480,14 @@ __device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer
 // Phase input staging (RMSNorm'd where the block says so), lane-permuted.
 // ---------------------------------------------------------------------------
 template <int B>
-__device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& sm, int kind, int layer, int s,
-                            int K, int tid_c) {
+__device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                            int s, int tid_c) {
+  const int kind = ph.kind, layer = ph.layer;
   const int cta = blockIdx.x, C = p.n_ctas;
   const int warp = tid_c >> 5, lane = tid_c & 31;
-  const int KP = round256(K);
+  // K: this segment's columns [k0, k0 + K) of the full input width KF
+  const int K = ph.K, KP = ph.KP, k0 = ph.k0, KF = ph.ldw;
+  if (ph.seg > 0) named_bar_sync(1, kNCT);   // every warp is done with the previous segment
   if (kind == PH_O && p.fuse_att) {
     // every CTA computes all heads (small attention): o lands directly in xin
     for (int b = 0; b < B; ++b)
@@ -451,27 +504,29 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
   const uint16_t* emb = nullptr;   // layer-0 input: the embedding rows of the tokens
   const float* src = nullptr;
   if (kind == PH_QKV && layer == 0) {
-    // input token: prompt for s < P, else the argmax of step s-1 (reduced from
-    // the per-CTA candidates, identically in every CTA).
-    if (tid_c < B) {
-      int tok;
-      if (s < p.P) {
-        tok = p.prompt[tid_c * p.P + s];
-      } else {
-        unsigned long long best = 0;
-        for (int c = 0; c < C; ++c) {
-          const unsigned long long v = p.cand[c * B + tid_c];
-          best = v > best ? v : best;
+    if (ph.seg == 0) {
+      // input token: prompt for s < P, else the argmax of step s-1 (reduced from
+      // the per-CTA candidates, identically in every CTA).
+      if (tid_c < B) {
+        int tok;
+        if (s < p.P) {
+          tok = p.prompt[tid_c * p.P + s];
+        } else {
+          unsigned long long best = 0;
+          for (int c = 0; c < C; ++c) {
+            const unsigned long long v = p.cand[c * B + tid_c];
+            best = v > best ? v : best;
+          }
+          tok = (int)argmax_key_index(best);
+          if (cta == 0) {
+            p.tokens[tid_c * p.G + (s - p.P)] = tok;
+            __threadfence_system();   // ordered before the completion flag
+          }
         }
-        tok = (int)argmax_key_index(best);
-        if (cta == 0) {
-          p.tokens[tid_c * p.G + (s - p.P)] = tok;
-          __threadfence_system();   // ordered before the completion flag
-        }
+        sm.tok[tid_c] = tok;
       }
-      sm.tok[tid_c] = tok;
+      named_bar_sync(1, kNCT);
     }
-    named_bar_sync(1, kNCT);
     emb = p.embed;
     gain = p.w_layers + p.off_gattn;
   } else {
@@ -483,13 +538,13 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
   // Inputs are read once into registers (up to kRegVals per thread), then the
   // RMSNorm scale is applied on the way into the lane-permuted smem layout.
   constexpr int kRegVals = 8;
-  const bool in_regs = (B == 1) && (KP <= kRegVals * kNCT);
+  const bool in_regs = (B == 1) && (ph.nseg == 1) && (KP <= kRegVals * kNCT);
   float rv[kRegVals];
   float inv[B];
 #pragma unroll
   for (int b = 0; b < B; ++b) inv[b] = 1.f;
-  auto load_in = [&](int b, int kk) -> float {
-    return emb ? bf16_bits_to_f32(emb[(size_t)sm.tok[b] * K + kk]) : src[b * K + kk];
+  auto load_in = [&](int b, int col) -> float {
+    return emb ? bf16_bits_to_f32(emb[(size_t)sm.tok[b] * KF + col]) : src[b * KF + col];
   };
   if (in_regs) {
 #pragma unroll
@@ -498,8 +553,9 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
       rv[i] = (kk < K) ? load_in(0, kk) : 0.f;
     }
   }
-  if (gain) {
-    // RMSNorm (normalise, then scale; eps inside the sqrt): fixed-order block sum.
+  if (gain && ph.seg == 0) {
+    // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt):
+    // fixed-order block sum; the scale is kept in smem for later K segments.
     float part[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) part[b] = 0.f;
@@ -511,7 +567,7 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
     } else {
 #pragma unroll
       for (int b = 0; b < B; ++b)
-        for (int kk = tid_c; kk < K; kk += kNCT) {
+        for (int kk = tid_c; kk < KF; kk += kNCT) {
           const float v = load_in(b, kk);
           part[b] = fmaf(v, v, part[b]);
         }
@@ -526,8 +582,12 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
     for (int b = 0; b < B; ++b) {
       float t = 0.f;
       for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + b];
-      inv[b] = 1.0f / sqrtf(t / (float)K + p.eps);
+      inv[b] = 1.0f / sqrtf(t / (float)KF + p.eps);
+      if (tid_c == 0) sm.inv[b] = inv[b];
     }
+  } else if (gain) {
+#pragma unroll
+    for (int b = 0; b < B; ++b) inv[b] = sm.inv[b];
   }
   if (in_regs) {
 #pragma unroll
@@ -548,9 +608,10 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
       for (int kk = tid_c; kk < KP; kk += kNCT) {
         float v = 0.f;
         if (kk < K) {
-          v = load_in(b, kk);
-          if (emb && cta == 0) p.x[b * p.d + kk] = v;
-          if (gain) v = v * inv[b] * bf16_bits_to_f32(gain[kk]);
+          const int col = k0 + kk;
+          v = load_in(b, col);
+          if (emb && cta == 0) p.x[b * p.d + col] = v;
+          if (gain) v = v * inv[b] * bf16_bits_to_f32(gain[col]);
         }
         sm.xin[xidx(b, kk, KP)] = v;
       }
@@ -759,7 +820,25 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
           for (int bb = 1; bb < B; ++bb)
             if (bb == b) v[q] = out[q][bb];
         }
-        switch (KIND) {
+        bool final_seg = true;
+        if (ph.nseg > 1) {
+          // split-K: kacc[b][row] holds the sum of the earlier segments (GU: gate
+          // and up interleaved); the last segment adds its part and goes on to
+          // the epilogue. Rows are owned by this CTA, so no atomics are needed.
+          float* acc = p.kacc + (size_t)b * ph.R * (gu ? 2 : 1);
+          final_seg = (ph.seg == ph.nseg - 1);
+#pragma unroll
+          for (int q = 0; q < NR; ++q)
+            if (has[q]) {
+              const int idx = gu ? 2 * (r + j0 + (q >> 1)) + (q & 1) : r + j0 + q;
+              const float t = (ph.seg == 0) ? v[q] : acc[idx] + v[q];
+              if (final_seg)
+                v[q] = t;
+              else
+                acc[idx] = t;
+            }
+        }
+        if (final_seg) switch (KIND) {
           case PH_QKV:
 #pragma unroll
             for (int q = 0; q < NR; ++q)
@@ -804,7 +883,7 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
       phase_bit ^= 1u;
     }
   }
-  if (KIND == PH_LM) {
+  if (KIND == PH_LM && ph.seg == ph.nseg - 1) {
     named_bar_sync(1, kNCT);
     if (tid_c < B) p.cand[cta * B + tid_c] = sm.best[tid_c];
   }
@@ -840,7 +919,7 @@ template <int B>
 __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams p, int n_stages,
                                                                    int kmax) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  const Smem sm = carve(smem_raw, n_stages, B, kmax);
+  const Smem sm = carve<B>(smem_raw, n_stages, kmax);
   const int warp_id = threadIdx.x >> 5;
   if (threadIdx.x == 0) {
     for (int i = 0; i < n_stages; ++i) {
@@ -854,7 +933,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
   __syncthreads();
 
   if (warp_id == 0) {
-    if ((threadIdx.x & 31) == 0) producer_loop(p, sm, n_stages);
+    if ((threadIdx.x & 31) == 0) producer_loop<B>(p, sm, n_stages);
     return;
   }
 
@@ -877,17 +956,20 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         c_att += t1 - t0;
         t0 = t1;
       } else {
-        const Phase ph = make_phase(p, kind, layer);
-        stage_input<B>(p, sm, kind, layer, s, ph.K, tid_c);
-        const long long t1 = clock64();
-        if (kind == PH_O && p.fuse_att)
-          c_att += t1 - t0;
-        else
-          c_stage += t1 - t0;
-        gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait, c_unit, c_units);
-        const long long t2 = clock64();
-        c_gemv += t2 - t1;
-        t0 = t2;
+        const int nseg = phase_segments<B>(p, kind);
+        for (int seg = 0; seg < nseg; ++seg) {
+          const Phase ph = make_phase<B>(p, kind, layer, seg);
+          stage_input<B>(p, sm, ph, s, tid_c);
+          const long long t1 = clock64();
+          if (kind == PH_O && p.fuse_att)
+            c_att += t1 - t0;
+          else
+            c_stage += t1 - t0;
+          gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait, c_unit, c_units);
+          const long long t2 = clock64();
+          c_gemv += t2 - t1;
+          t0 = t2;
+        }
       }
       target += (unsigned long long)p.n_ctas;
       grid_barrier(p, target, tid_c);

@@ -25,7 +25,19 @@ constexpr int kAttHd = 128;             // max attention head_dim
 constexpr int kMaxUnits = 128;          // (row, 256-col chunk) work units per tile
 constexpr int kMaxCtas = 160;           // >= 148 SMs
 constexpr int kMaxSeqCap = 512;         // attention keeps <= 16 scores per lane
-constexpr int kXinBytesCap = 96 * 1024; // activation staging (B * K * 4)
+constexpr int kXinSegBytes = 64 * 1024; // activation staging per K segment (B * cols * 4)
+// Columns of one K segment for batch B: phases whose B*K*4 exceeds the staging
+// capacity run as several K segments (split-K inside the owning CTA).
+#ifdef __CUDACC__
+#define MX_HD __host__ __device__
+#else
+#define MX_HD
+#endif
+MX_HD constexpr int decode_seg_cols(int B) { return (kXinSegBytes / (B * 4)) & ~255; }
+// Activation staging columns for the widest phase input kmax.
+MX_HD constexpr int decode_xin_cols(int B, int kmax) {
+  return ((kmax + 255) & ~255) < decode_seg_cols(B) ? ((kmax + 255) & ~255) : decode_seg_cols(B);
+}
 
 // One decode task on one partition: all P+G-1 steps in ONE persistent launch
 // (grid = the partition's SMs, one CTA per SM), phases separated by a
@@ -50,6 +62,7 @@ struct DecodeParams {
   float* o;                  // [B][q_dim]
   float* a;                  // [B][ff]
   unsigned long long* cand;  // [kMaxCtas][B] per-CTA argmax keys
+  float* kacc;               // split-K partial sums [B][2 * max(qkv_rows, ff, d, V)]
   uint16_t* kc;              // [L][B][Hkv][max_seq][hd] bf16
   uint16_t* vc;
   const int* prompt;         // [B][P] (host-mapped)

@@ -97,6 +97,7 @@ struct Lib {
 
 static std::mutex g_init_mu;
 static bool g_decode_prof = false;
+static bool g_trace_resize = false;   // MX_TRACE_RESIZE=1: per-resize timing on stderr
 static Lib* g_lib = nullptr;
 
 // ---------------------------------------------------------------------------
@@ -160,9 +161,9 @@ static int validate_fn(const mx_fn_desc& d) {
       return MX_EINVAL;
     }
     const int kmax = std::max(std::max(c.d_model, q), c.d_ff);
-    if ((int64_t)c.max_batch * ((kmax + 255) / 256 * 256) * 4 > mxk::kXinBytesCap ||
-        mxk::decode_smem_bytes(c.max_batch, kmax, nullptr) < 0) {
-      set_error("decode cfg: max_batch * max(d, q_dim, d_ff) * 4 > 96 KiB activation staging");
+    if (mxk::decode_smem_bytes(c.max_batch, kmax, nullptr) < 0) {
+      set_error("decode cfg: shared-memory plan does not fit (max_batch %d, K %d)", c.max_batch,
+                kmax);
       return MX_EINVAL;
     }
     if (!(c.rms_eps >= 0.f) || !(c.rope_theta > 0.f)) {
@@ -444,6 +445,8 @@ static int alloc_decode_slot(Partition& p, FnInst& fi, Slot& s) {
   if ((rc = alloc_ptr(p, B * q * 4, &s.o))) return rc;
   if ((rc = alloc_ptr(p, B * ff * 4, &s.a))) return rc;
   if ((rc = alloc_ptr(p, (uint64_t)mxk::kMaxCtas * B * 8, &s.cand))) return rc;
+  const uint64_t kacc_rows = std::max(std::max(q + 2 * kv, 2 * ff), std::max(d, V));
+  if ((rc = alloc_ptr(p, B * kacc_rows * 4, &s.kacc))) return rc;
   if ((rc = alloc_ptr(p, L * B * kv * T * 2, &s.kc))) return rc;
   if ((rc = alloc_ptr(p, L * B * kv * T * 2, &s.vc))) return rc;
   if ((rc = alloc_ptr(p, B * T * 4, &s.prompt))) return rc;
@@ -622,6 +625,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.o = reinterpret_cast<float*>(s.o);
     k.a = reinterpret_cast<float*>(s.a);
     k.cand = reinterpret_cast<unsigned long long*>(s.cand);
+    k.kacc = reinterpret_cast<float*>(s.kacc);
     k.kc = reinterpret_cast<uint16_t*>(s.kc);
     k.vc = reinterpret_cast<uint16_t*>(s.vc);
     k.prompt = reinterpret_cast<const int*>(s.d_in);
@@ -941,6 +945,7 @@ static int init_impl(const std::vector<int>& ordinals) {
   if (g_lib) return MX_OK;
   setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
   g_decode_prof = getenv("MX_DECODE_PROF") && atoi(getenv("MX_DECODE_PROF")) == 1;
+  g_trace_resize = getenv("MX_TRACE_RESIZE") && atoi(getenv("MX_TRACE_RESIZE")) == 1;
   if (const char* e = getenv("MX_INFLIGHT")) {
     const int v = atoi(e);
     g_inflight_override = (v == 1 || v == 2) ? (size_t)v : 0;
@@ -1219,12 +1224,16 @@ mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
   const SchedPart& sp = L->sched->part(part);
   const bool same_sms = sp.shared || (groups == sp.groups && whole == sp.whole);
   std::unique_ptr<Exec> ne;
+  const uint64_t t0 = now_ns();
   if (!same_sms) {
     rc = make_exec(g, groups, whole, sp.epoch + 1, &ne);
     if (rc) return rc;
   }
+  const uint64_t t1 = now_ns();
+  uint64_t t2 = 0;
   {
     std::lock_guard<std::mutex> glk(g.mu);
+    t2 = now_ns();
     if (ne) {
       // FIFO across the switch: the new stream starts after the old one's last work.
       Exec* old = p.cur.get();
@@ -1245,6 +1254,10 @@ mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
     }
     p.arena.set_quota(quota);
   }
+  if (g_trace_resize)
+    fprintf(stderr, "[mx] part_resize(%d -> %d SMs): new exec %.3f ms, dispatcher lock %.3f ms, "
+            "switch %.3f ms\n", part, smc, (t1 - t0) * 1e-6, (t2 - t1) * 1e-6,
+            (now_ns() - t2) * 1e-6);
   rc = L->sched->resize(part, sm_count, hbm_bytes);
   return rc;
 }

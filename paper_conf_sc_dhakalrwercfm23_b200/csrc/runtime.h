@@ -79,7 +79,7 @@ struct Task {
 struct Slot {
   bool busy = false;
   // decode
-  CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
+  CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kacc = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
               logits = 0;
   // mpnn
   CUdeviceptr atom_off = 0, atom_type = 0, edge_off = 0, edges = 0, out = 0, tile_off = 0;

@@ -113,6 +113,8 @@ def test_task_validation_rejects_bad_inputs():
     too_long = mx.decode_task(1, np.zeros((1, 60), dtype=np.int32), 8)   # 67 > max_seq 64
     with pytest.raises(mx.MxError):
         mx.task_default_cost(desc, too_long)
-    big = mx.decode_desc(LLAMA7B, max_batch=4)   # 4 * 11008 * 4 > 96 KiB staging
+    big = mx.decode_desc(LLAMA7B, max_batch=8)   # split-K: wide inputs at batch 8 are valid
+    assert mx.task_default_cost(big, mx.decode_task(1, np.zeros((8, 4), dtype=np.int32), 4)) > 0
+    over = mx.decode_desc(LLAMA7B, max_batch=9)  # batch > 8
     with pytest.raises(mx.MxError):
-        mx.task_default_cost(big, mx.decode_task(1, np.zeros((4, 4), dtype=np.int32), 4))
+        mx.task_default_cost(over, mx.decode_task(1, np.zeros((9, 4), dtype=np.int32), 4))

@@ -9,7 +9,7 @@ import pytest
 from oracle import decode as od
 from oracle import mpnn as om
 from oracle import sched as S
-from workloads.configs import TINY, GPT2S, RAGGED, LLAMA7B, MPNN
+from workloads.configs import TINY, GPT2S, RAGGED, LLAMA7B, MPNN, SPLITK
 from workloads.inputs import prompt_tokens, molecules
 from workloads.weights import decode_weights, mpnn_weights
 
@@ -102,6 +102,40 @@ def test_results_identical_across_partition_sizes(mxlib, parts):
         assert np.array_equal(lg.view(np.uint32), outs[0][1].view(np.uint32))
 
 
+def test_shared_partitions_time_share_and_concurrent(mxlib):
+    """N1 modes (unpartitioned streams, cooperative launches): two time-shared
+    streams (148-CTA grids competing for every SM) and two concurrent ones
+    (74-CTA grids) give outputs bit-identical to a green-context partition."""
+    cfg = TINY
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg))
+    ref_p = mxlib.part_create(0, 16, 256 << 20)
+    prompts = [prompt_tokens(20 + k, 1, 8, cfg.vocab) for k in range(6)]
+    ref = []
+    for pr in prompts:
+        t = mxlib.decode_task(fn, pr, 10, want_logits=True, vocab=cfg.vocab)
+        mxlib.fn_submit(ref_p, t)
+        assert mxlib.fn_wait(t)["status"] == 0
+        ref.append((t.tokens.copy(), t.logits.copy()))
+    mxlib.part_destroy(ref_p)
+    for grid in (148, 74):
+        sp = [mxlib.part_create_shared(0, grid, 256 << 20) for _ in range(2)]
+        info = mxlib.part_query(sp[0])
+        assert info["shared"] == 1 and info["group_mask"] == 0 and info["n_ctas"] == grid
+        ts = []
+        for k, pr in enumerate(prompts):
+            t = mxlib.decode_task(fn, pr, 10, want_logits=(k % 2 == 0), vocab=cfg.vocab)
+            mxlib.fn_submit(sp[k % 2], t)
+            ts.append(t)
+        for k, t in enumerate(ts):
+            r = mxlib.fn_wait(t)
+            assert r["status"] == 0, r
+            assert np.array_equal(t.tokens, ref[k][0])
+            if k % 2 == 0:
+                assert np.array_equal(t.logits.view(np.uint32), ref[k][1].view(np.uint32))
+        for p in sp:
+            mxlib.part_destroy(p)
+
+
 def test_c2_gpt2s_one_task_full_size(mxlib, parts):
     """configs[1] shape at full size (12 layers, d=768, V=50257, P=16, G=32)."""
     cfg = GPT2S
@@ -129,6 +163,36 @@ def test_c3_llama7b_width_two_layers(mxlib, parts):
     mxlib.fn_submit(p, t)
     assert mxlib.fn_wait(t)["status"] == 0
     _check_decode(cfg, w, prompt, 3, t.tokens, t.logits)
+
+
+def test_split_k_batch8_ragged_segments(mxlib, parts):
+    """Split-K (inputs wider than the 64 KiB activation staging at batch 8):
+    d_model 2056 and d_ff 2600 run as 2 K segments each, the second ragged;
+    GQA, separate attention phase. Also batch 3 on the same instance."""
+    cfg = SPLITK
+    p = parts(20, hbm=1 << 30)
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=8))
+    w = decode_weights(cfg)
+    for B, P, G in ((8, 5, 4), (3, 3, 3)):
+        prompt = prompt_tokens(31 + B, B, P, cfg.vocab)
+        t = mxlib.decode_task(fn, prompt, G, want_logits=True, vocab=cfg.vocab)
+        mxlib.fn_submit(p, t)
+        assert mxlib.fn_wait(t)["status"] == 0
+        rel = _check_decode(cfg, w, prompt, G, t.tokens, t.logits)
+        print(f"split-K B={B}: max rel err {rel:.2e}")
+
+
+def test_c3_llama7b_width_batch8(mxlib, parts):
+    """configs[2] widths at batch 8 (every phase but O runs split-K), 2 layers."""
+    cfg = LLAMA7B.with_layers(2)
+    p = parts(48, hbm=4 << 30)
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=8))
+    w = decode_weights(cfg)
+    prompt = prompt_tokens(3, 8, 3, cfg.vocab)
+    t = mxlib.decode_task(fn, prompt, 2, want_logits=True, vocab=cfg.vocab)
+    mxlib.fn_submit(p, t)
+    assert mxlib.fn_wait(t)["status"] == 0
+    _check_decode(cfg, w, prompt, 2, t.tokens, t.logits)
 
 
 def test_mpnn_parity(mxlib, parts):

@@ -259,8 +259,9 @@ def cmd_c5(a, mx):
     mfl = float(np.mean([mpnn_task_flops(m, MPNN.hidden, MPNN.steps) for m in mol_cache]))
     out = {"suite": "D5 c5", "workload": f"configs[4]: task farm of {a.tasks} tasks, 50/50 "
            "GPT-2s decode / MPNN, shuffled (seed 42), WLAW over 7 fill partitions, layout "
-           f"alternating fill-7 <-> {LAYOUT_B} via part_resize after every {a.resize_every} "
-           "submissions", "peak_gbs": peak_gbs()}
+           f"alternating fill-7 <-> {LAYOUT_B} via part_resize between waves of "
+           f"{a.resize_every} submissions (wave w+2 is submitted after wave w completes)",
+           "peak_gbs": peak_gbs()}
     A = LAYOUTS_FILL[7]
     for label, sizes, n_tasks in (("partitioned", A, a.tasks), ("1_partition", [148], a.base_tasks)):
         parts = [mx.part_create(0, s, 1 << 30) for s in sizes]
@@ -273,12 +274,25 @@ def cmd_c5(a, mx):
         resize_ms = []
         h0 = time.perf_counter()
         use_b = False
-        for i, (_, t) in enumerate(items):
-            if label == "partitioned" and i > 0 and i % a.resize_every == 0:
-                use_b = not use_b
-                resize_ms += apply_layout(mx, parts, LAYOUT_B if use_b else A)
-            mx.fn_submit(mx.MX_PART_ANY, t)
-        res = [mx.fn_wait(t) for _, t in items]
+        # Waves of `resize_every` submissions. Before wave w >= 2 is submitted,
+        # wave w-2 is collected and the layout flips, so every resize happens
+        # while about one wave of work is queued or running (a resize between
+        # instantaneous submissions would only ever see an idle queue).
+        W = a.resize_every
+        waves = [items[i:i + W] for i in range(0, len(items), W)]
+        res_by_wave = {}
+        for w, wave in enumerate(waves):
+            if w >= 2:
+                res_by_wave[w - 2] = [mx.fn_wait(t) for _, t in waves[w - 2]]
+                if label == "partitioned":
+                    use_b = not use_b
+                    resize_ms += apply_layout(mx, parts, LAYOUT_B if use_b else A)
+            for _, t in wave:
+                mx.fn_submit(mx.MX_PART_ANY, t)
+        for w in range(len(waves)):
+            if w not in res_by_wave:
+                res_by_wave[w] = [mx.fn_wait(t) for _, t in waves[w]]
+        res = [r for w in range(len(waves)) for r in res_by_wave[w]]
         wall = time.perf_counter() - h0
         assert all(r["status"] == 0 for r in res)
         st = class_stats(res, [k for k, _ in items], mfl, n_tasks // 2, n_tasks - n_tasks // 2)

@@ -67,9 +67,15 @@ LLAMA7B = DecodeCfg("llama7b", n_layers=32, d_model=4096, n_heads=32, n_kv_heads
 RAGGED = DecodeCfg("ragged", n_layers=2, d_model=264, n_heads=6, n_kv_heads=2, head_dim=32,
                    d_ff=712, vocab=1031, seed=0x5EED)
 
+# split-K shape used only by parity tests: at batch 8 the inputs of width d_model
+# (2056 -> 2 segments, ragged second) and d_ff (2600 -> 2 segments) exceed the
+# 64 KiB activation staging, q_dim 512 does not; GQA 8/2, separate attention phase
+SPLITK = DecodeCfg("splitk", n_layers=2, d_model=2056, n_heads=8, n_kv_heads=2, head_dim=64,
+                   d_ff=2600, vocab=1031, seed=0x5A17)
+
 MPNN = MpnnCfg()
 
-DECODE_CFGS = {c.name: c for c in (TINY, GPT2S, LLAMA7B, RAGGED)}
+DECODE_CFGS = {c.name: c for c in (TINY, GPT2S, LLAMA7B, RAGGED, SPLITK)}
 
 # Default seeds
 SEED_PROMPT = 0xC0FFEE
