@@ -14,7 +14,7 @@ template <int B>
 int set_attrs_b(int device);
 
 int decode_smem_bytes(int B, int kmax, int* n_stages) {
-  const int fixed = B * decode_xin_cols(B, kmax) * 4 + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 +
+  const int fixed = decode_xin_bytes(B, kmax) + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 +
                     8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 128;
   const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
   const int cap = 227 * 1024;
@@ -25,7 +25,11 @@ int decode_smem_bytes(int B, int kmax, int* n_stages) {
   return ns * per_stage + fixed;
 }
 
-int decode_fuse_attention(int B, int H, int hd) { return (B * H * hd <= 1024) ? 1 : 0; }
+// Fused (per-CTA) attention only for small attention on the CUDA-core path
+// (the tensor-core path stages its activations as bf16 hi/lo, not fp32).
+int decode_fuse_attention(int B, int H, int hd) {
+  return (B < kTcMinBatch && B * H * hd <= 1024) ? 1 : 0;
+}
 
 uint64_t decode_barriers(int L, int P, int G, int fuse_att) {
   const uint64_t S = (uint64_t)(P + G - 1);

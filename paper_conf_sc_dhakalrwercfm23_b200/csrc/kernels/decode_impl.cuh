@@ -49,6 +49,21 @@ constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
 #define MX_FULL_WAIT(b, ph) mbar_try_wait_sleep(b, ph, 20000u)
 #define MX_EMPTY_WAIT(b, ph) mbar_try_wait_sleep(b, ph, 20000u)
 #endif
+// Bounded mbarrier wait: a launch that would otherwise hang (a protocol error
+// or a failed copy) raises *err after 4 s and stops waiting, so the task
+// completes with MX_EDEVICE instead of wedging its partition.
+__device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity, int* err) {
+  if (MX_FULL_WAIT(bar, parity)) return;
+  const uint64_t t0 = globaltimer();
+  while (!MX_FULL_WAIT(bar, parity)) {
+    if (ld_volatile_i32(err)) return;
+    if (globaltimer() - t0 > 4000000000ull) {
+      atomicExch(err, 1);
+      return;
+    }
+  }
+}
+
 constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
 
 // One GEMV phase, or one K segment of it. Phases whose staged activations
@@ -58,6 +73,8 @@ constexpr int kCPG = 8;                     // 256-column chunks per GEMV work u
 // to the slot's kacc buffer, and the last segment applies the epilogue to
 // (kacc + partial). Segment widths depend only on the shape, so results stay
 // independent of the partition size.
+constexpr int kTcRows = 8;   // weight rows per tensor-core tile (the n of mma.m16n8k16)
+
 struct Phase {
   int kind, layer, R, K, KP, NC, NG, TR;
   int ldw;         // row stride of the weight matrix in HBM (= the full K)
@@ -87,10 +104,23 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
     default: break;
   }
   ph.ldw = K;
+  ph.seg = seg;
+  if constexpr (B >= kTcMinBatch) {
+    // tensor-core path: K segments of <= kTcCols columns (multiples of 32), one
+    // tile = 8 weight rows (GU: 4 gate + 4 up) x the segment = one stage
+    ph.nseg = max(1, (K + kTcCols - 1) / kTcCols);
+    const int w = (((K + ph.nseg - 1) / ph.nseg) + 31) & ~31;
+    ph.k0 = seg * w;
+    ph.K = min(w, K - ph.k0);
+    ph.KP = (ph.K + 31) & ~31;
+    ph.NC = 1;
+    ph.NG = 1;
+    ph.TR = (kind == PH_GU) ? kTcRows / 2 : kTcRows;
+    return ph;
+  }
   constexpr int KS = decode_seg_cols(B);
   ph.nseg = (K + KS - 1) / KS;
   if (ph.nseg < 1) ph.nseg = 1;
-  ph.seg = seg;
   if (ph.nseg > 1) {
     const int w = round256((K + ph.nseg - 1) / ph.nseg);
     ph.k0 = seg * w;
@@ -116,7 +146,7 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
 template <int B>
 __device__ __forceinline__ int phase_segments(const DecodeParams& p, int kind) {
   const int K = (kind == PH_O) ? p.q_dim : (kind == PH_DOWN) ? p.ff : p.d;
-  constexpr int KS = decode_seg_cols(B);
+  constexpr int KS = (B >= kTcMinBatch) ? kTcCols : decode_seg_cols(B);
   return kind == PH_ATT ? 1 : max(1, (K + KS - 1) / KS);
 }
 
@@ -157,6 +187,7 @@ struct Smem {
   int* tok;                  // [8]
   float* wsum;               // [kConsumerWarps][8]
   float* inv;                // [8] RMSNorm scale of the phase input (kept across K segments)
+  uint8_t* zero;             // [64] zeros (tensor-core path)
 };
 
 template <int B>
@@ -166,7 +197,8 @@ __device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int kmax) {
   s.ring = p;
   p += (size_t)n_stages * kStageBytes;
   s.xin = reinterpret_cast<float*>(p);
-  p += (size_t)B * decode_xin_cols(B, kmax) * 4;
+  p += (size_t)decode_xin_bytes(B, kmax);
+  s.zero = p - 64;   // tensor-core path: 64 zero bytes (ldmatrix rows of absent sequences)
   s.red = reinterpret_cast<float*>(p);
   p += (size_t)n_stages * kMaxUnits * B * 4;
   s.cnt = reinterpret_cast<int*>(p);
@@ -264,14 +296,24 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
           // never abandons the stream: after a barrier timeout the consumers run
           // through the remaining phases without waiting, so every slot is freed.
           const long long tw = clock64();
-          while (!MX_EMPTY_WAIT(&sm.empty[stage], phase_bit ^ 1u)) {
-          }
+          mbar_wait_bounded(&sm.empty[stage], phase_bit ^ 1u, p.err);
           wait_cyc += clock64() - tw;
           const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
           const uint32_t total = (kind == PH_GU) ? 2u * one : one;
           uint8_t* dst = sm.ring + (size_t)stage * kStageBytes;
           mbar_arrive_expect_tx(&sm.full[stage], total);
-          if (ph.nseg == 1) {
+          if constexpr (B >= kTcMinBatch) {
+            // tensor-core tile: rows at a padded stride (conflict-free ldmatrix);
+            // GU: gate rows 0..3, up rows 4..7
+            const uint32_t rb = (uint32_t)ph.K * 2u, ws = (uint32_t)ph.KP * 2u + 16u;
+            for (int i = 0; i < n; ++i) {
+              const size_t src = (size_t)(r + i) * ph.ldw + ph.k0;
+              bulk_g2s_evict_first(dst + i * ws, ph.w0 + src, rb, &sm.full[stage], pol);
+              if (kind == PH_GU)
+                bulk_g2s_evict_first(dst + (kTcRows / 2 + i) * ws, ph.w1 + src, rb,
+                                     &sm.full[stage], pol);
+            }
+          } else if (ph.nseg == 1) {
             // whole rows: one contiguous copy per matrix
             bulk_g2s_evict_first(dst, ph.w0 + (size_t)r * ph.K, one, &sm.full[stage], pol);
             if (kind == PH_GU)
@@ -479,6 +521,26 @@ __device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer
 // ---------------------------------------------------------------------------
 // Phase input staging (RMSNorm'd where the block says so), lane-permuted.
 // ---------------------------------------------------------------------------
+// Strided loop over [0, n) with U independent loads in flight per thread (the
+// inputs come from L2, ~1 us away: a plain loop would serialise them).
+template <int U, typename Load, typename Use>
+__device__ __forceinline__ void batched_loop(int n, int tid, int stride, Load load, Use use) {
+  using V = decltype(load(0));
+  for (int base = tid; base < n; base += U * stride) {
+    V v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int i = base + u * stride;
+      if (i < n) v[u] = load(i);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int i = base + u * stride;
+      if (i < n) use(i, v[u]);
+    }
+  }
+}
+
 template <int B>
 __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                             int s, int tid_c) {
@@ -540,11 +602,14 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
   constexpr int kRegVals = 8;
   const bool in_regs = (B == 1) && (ph.nseg == 1) && (KP <= kRegVals * kNCT);
   float rv[kRegVals];
-  float inv[B];
-#pragma unroll
-  for (int b = 0; b < B; ++b) inv[b] = 1.f;
   auto load_in = [&](int b, int col) -> float {
     return emb ? bf16_bits_to_f32(emb[(size_t)sm.tok[b] * KF + col]) : src[b * KF + col];
+  };
+  // staged column kk of the segment: (input, gain) loaded together
+  auto load_staged = [&](int b, int kk) -> float2 {
+    if (kk >= K) return make_float2(0.f, 0.f);
+    const int col = k0 + kk;
+    return make_float2(load_in(b, col), gain ? bf16_bits_to_f32(gain[col]) : 1.f);
   };
   if (in_regs) {
 #pragma unroll
@@ -556,40 +621,49 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
   if (gain && ph.seg == 0) {
     // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt):
     // fixed-order block sum; the scale is kept in smem for later K segments.
-    float part[B];
-#pragma unroll
-    for (int b = 0; b < B; ++b) part[b] = 0.f;
     if (in_regs) {
+      float acc = 0.f;
 #pragma unroll
-      for (int i = 0; i < kRegVals; ++i) {
-        part[0] = fmaf(rv[i], rv[i], part[0]);
-      }
+      for (int i = 0; i < kRegVals; ++i) acc = fmaf(rv[i], rv[i], acc);
+      acc = warp_sum(acc);
+      if (lane == 0) sm.wsum[warp * 8] = acc;
     } else {
-#pragma unroll
-      for (int b = 0; b < B; ++b)
-        for (int kk = tid_c; kk < KF; kk += kNCT) {
-          const float v = load_in(b, kk);
-          part[b] = fmaf(v, v, part[b]);
-        }
-    }
-#pragma unroll
-    for (int b = 0; b < B; ++b) {
-      part[b] = warp_sum(part[b]);
-      if (lane == 0) sm.wsum[warp * 8 + b] = part[b];
+      for (int b = 0; b < B; ++b) {
+        float acc = 0.f;
+        batched_loop<4>(KF, tid_c, kNCT, [&](int kk) { return load_in(b, kk); },
+                        [&](int, float v) { acc = fmaf(v, v, acc); });
+        acc = warp_sum(acc);
+        if (lane == 0) sm.wsum[warp * 8 + b] = acc;
+      }
     }
     named_bar_sync(1, kNCT);
-#pragma unroll
-    for (int b = 0; b < B; ++b) {
+    if (tid_c < B) {
       float t = 0.f;
-      for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + b];
-      inv[b] = 1.0f / sqrtf(t / (float)KF + p.eps);
-      if (tid_c == 0) sm.inv[b] = inv[b];
+      for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + tid_c];
+      sm.inv[tid_c] = 1.0f / sqrtf(t / (float)KF + p.eps);
     }
-  } else if (gain) {
-#pragma unroll
-    for (int b = 0; b < B; ++b) inv[b] = sm.inv[b];
+    named_bar_sync(1, kNCT);
   }
-  if (in_regs) {
+  if constexpr (B >= kTcMinBatch) {
+    // tensor-core operand: x = hi + lo (bf16 pair), rows [b][KP + 8] (padded)
+    uint16_t* xh = reinterpret_cast<uint16_t*>(sm.xin);
+    uint16_t* xl = xh + B * (KP + 8);
+    for (int b = 0; b < B; ++b) {
+      const float ib = gain ? sm.inv[b] : 1.f;
+      batched_loop<4>(KP, tid_c, kNCT, [&](int kk) { return load_staged(b, kk); },
+                      [&](int kk, float2 xg) {
+                        float v = 0.f;
+                        if (kk < K) {
+                          v = xg.x;
+                          if (emb && cta == 0) p.x[b * p.d + k0 + kk] = v;
+                          if (gain) v = v * ib * xg.y;
+                        }
+                        const uint16_t h = f32_to_bf16_rne(v);
+                        xh[b * (KP + 8) + kk] = h;
+                        xl[b * (KP + 8) + kk] = f32_to_bf16_rne(v - bf16_bits_to_f32(h));
+                      });
+    }
+  } else if (in_regs) {
 #pragma unroll
     for (int i = 0; i < kRegVals; ++i) {
       const int kk = tid_c + i * kNCT;
@@ -597,24 +671,24 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
         float v = rv[i];
         if (kk < K) {
           if (emb && cta == 0) p.x[kk] = v;
-          if (gain) v = v * inv[0] * bf16_bits_to_f32(gain[kk]);
+          if (gain) v = v * sm.inv[0] * bf16_bits_to_f32(gain[kk]);
         }
         sm.xin[xidx(0, kk, KP)] = v;
       }
     }
   } else {
-#pragma unroll
     for (int b = 0; b < B; ++b) {
-      for (int kk = tid_c; kk < KP; kk += kNCT) {
-        float v = 0.f;
-        if (kk < K) {
-          const int col = k0 + kk;
-          v = load_in(b, col);
-          if (emb && cta == 0) p.x[b * p.d + col] = v;
-          if (gain) v = v * inv[b] * bf16_bits_to_f32(gain[col]);
-        }
-        sm.xin[xidx(b, kk, KP)] = v;
-      }
+      const float ib = gain ? sm.inv[b] : 1.f;
+      batched_loop<4>(KP, tid_c, kNCT, [&](int kk) { return load_staged(b, kk); },
+                      [&](int kk, float2 xg) {
+                        float v = 0.f;
+                        if (kk < K) {
+                          v = xg.x;
+                          if (emb && cta == 0) p.x[b * p.d + k0 + kk] = v;
+                          if (gain) v = v * ib * xg.y;
+                        }
+                        sm.xin[xidx(b, kk, KP)] = v;
+                      });
     }
   }
   named_bar_sync(1, kNCT);
@@ -743,8 +817,7 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
     // every warp observes the stage fill before releasing it (keeps the empty
     // barrier's arrival count per round exact)
     const long long tw = clock64();
-    while (!MX_FULL_WAIT(&sm.full[stage], phase_bit)) {
-    }
+    mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
     wait_cyc += clock64() - tw;
     const uint16_t* wt = reinterpret_cast<const uint16_t*>(sm.ring + (size_t)stage * kStageBytes);
     float* red = sm.red + (size_t)stage * kMaxUnits * B;
@@ -889,6 +962,171 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
   }
 }
 
+// ---------------------------------------------------------------------------
+// Tensor-core GEMV (K7, batch >= kTcMinBatch): at batch 4-8 the CUDA-core unit
+// is shared-memory bound (each weight needs B fp32 activations), so the GEMV
+// runs as mma.sync.m16n8k16: A = activations (rows = sequences, only the first
+// B of 16 real; the rest point at a zero block), B = 8 weight rows of the tile
+// ("col" operand = the row-major weight rows), fp32 accumulate. Activations are
+// fed as a bf16 hi/lo pair (two MMAs, ~16-bit mantissa, reading A17); weights
+// are exact in bf16. One tile (8 rows x one K segment) is one stage and is
+// consumed entirely by its owner warp (row group g -> warp g % 12), with four
+// independent accumulator chains summed in a fixed order at the end.
+// D fragment: lane (g, t) holds sequence g, tile rows 2t and 2t+1.
+// ---------------------------------------------------------------------------
+template <int B, int KIND>
+__device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem& sm,
+                                              const Phase& ph, int k, int s, int tid_c,
+                                              uint32_t& stage, uint32_t& phase_bit, int n_stages,
+                                              long long& wait_cyc, long long& unit_cyc,
+                                              long long& unit_cnt) {
+  const int C = p.n_ctas, cta = blockIdx.x;
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int g8 = lane >> 2, t4 = lane & 3;
+  const int lr = lane & 7, lm = lane >> 3;
+  constexpr bool gu = (KIND == PH_GU);
+  const int K = ph.K, KP = ph.KP;
+  const uint32_t ws = (uint32_t)KP * 2u + 16u;   // weight / activation row stride (bytes)
+  const uint32_t xh = smem_u32(sm.xin);
+  const uint32_t xl = xh + (uint32_t)B * ws;
+  const uint32_t zero = smem_u32(sm.zero);
+  // per-lane ldmatrix row addresses (row lr of matrix lm = columns 8*lm..8*lm+7)
+  const bool arow = lr < B;
+  const uint32_t a_hi = arow ? xh + (uint32_t)lr * ws + (uint32_t)lm * 16u : zero;
+  const uint32_t a_lo = arow ? xl + (uint32_t)lr * ws + (uint32_t)lm * 16u : zero;
+  const uint32_t a_step = arow ? 64u : 0u;   // 32 columns per iteration
+  const bool last_seg = (ph.seg == ph.nseg - 1);
+  int r0, r1;
+  my_rows(ph.R, C, cta, k, &r0, &r1);
+  if (KIND == PH_LM) {
+    if (tid_c < B) sm.best[tid_c] = 0ull;
+    named_bar_sync(1, kNCT);
+  }
+  int gidx = 0;
+  for (int r = r0; r < r1; r += ph.TR, ++gidx) {
+    // Every warp observes every stage fill and arrives on its empty barrier
+    // (count kConsumerWarps): a parity wait only tells two consecutive phases
+    // apart, so no warp may skip stages and run a full ring ahead. Only the
+    // owner warp computes the tile.
+    const long long tw = clock64();
+    mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
+    const long long tu = clock64();
+    wait_cyc += tu - tw;
+    if (gidx % kConsumerWarps != warp) {
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.empty[stage]);
+    } else {
+      const int n = min(ph.TR, r1 - r);
+      const uint32_t wt = smem_u32(sm.ring + (size_t)stage * kStageBytes) + (uint32_t)lr * ws +
+                          (uint32_t)lm * 16u;
+      float acc[4][4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[c][j] = 0.f;
+      uint32_t ah = a_hi, al = a_lo, wp = wt;
+      for (int kk = 0; kk < K; kk += 32) {
+        uint32_t w0, w1, w2, w3, h0, h1, h2, h3, l0, l1, l2, l3;
+        ldsm_x4(wp, w0, w1, w2, w3);
+        ldsm_x4(ah, h0, h1, h2, h3);
+        ldsm_x4(al, l0, l1, l2, l3);
+        if (kk + 32 > K) {
+          // ragged end: weight columns >= K hold stale data -> zero their fragments
+          // (b0: k = 2t, 2t+1; b1: k = 8 + 2t, 8 + 2t + 1 of each 16-column step)
+          const int kb = kk + 2 * t4;
+          if (kb >= K) w0 = 0u;
+          if (kb + 8 >= K) w1 = 0u;
+          if (kb + 16 >= K) w2 = 0u;
+          if (kb + 24 >= K) w3 = 0u;
+        }
+        mma_bf16(acc[0], h0, 0u, h1, 0u, w0, w1);
+        mma_bf16(acc[1], l0, 0u, l1, 0u, w0, w1);
+        mma_bf16(acc[2], h2, 0u, h3, 0u, w2, w3);
+        mma_bf16(acc[3], l2, 0u, l3, 0u, w2, w3);
+        wp += 64u;
+        ah += a_step;
+        al += a_step;
+      }
+      float v0 = (acc[0][0] + acc[1][0]) + (acc[2][0] + acc[3][0]);
+      float v1 = (acc[0][1] + acc[1][1]) + (acc[2][1] + acc[3][1]);
+      // all smem reads of the tile are done: release the stage to the producer
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sm.empty[stage]);
+      if (gu) {
+        // tile rows 0..3 = gate rows, 4..7 = up rows: lanes t4 < 2 (gate) fetch
+        // the matching up values from lane ^ 2
+        const float u0 = __shfl_xor_sync(0xffffffffu, v0, 2);
+        const float u1 = __shfl_xor_sync(0xffffffffu, v1, 2);
+        if (g8 < B && t4 < 2) {
+          const int b = g8;
+          float gv[2] = {v0, v1}, uv[2] = {u0, u1};
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int j = 2 * t4 + e;
+            if (j >= n) continue;
+            const int row = r + j;
+            float gt = gv[e], up = uv[e];
+            if (ph.nseg > 1) {
+              float* acc_g = p.kacc + (size_t)b * ph.R * 2 + 2 * row;
+              if (ph.seg > 0) {
+                gt += acc_g[0];
+                up += acc_g[1];
+              }
+              if (!last_seg) {
+                acc_g[0] = gt;
+                acc_g[1] = up;
+                continue;
+              }
+            }
+            p.a[b * p.ff + row] = gt / (1.0f + expf(-gt)) * up;
+          }
+        }
+      } else if (g8 < B) {
+        const int b = g8;
+        float vv[2] = {v0, v1};
+        unsigned long long kb = 0ull;
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int j = 2 * t4 + e;
+          if (j >= n) continue;
+          const int row = r + j;
+          float v = vv[e];
+          if (ph.nseg > 1) {
+            float* acc_r = p.kacc + (size_t)b * ph.R + row;
+            if (ph.seg > 0) v += *acc_r;
+            if (!last_seg) {
+              *acc_r = v;
+              continue;
+            }
+          }
+          switch (KIND) {
+            case PH_QKV: p.qkv[b * p.qkv_rows + row] = v; break;
+            case PH_O:
+            case PH_DOWN: p.x[b * p.d + row] += v; break;
+            case PH_LM: {
+              const unsigned long long kq = argmax_key(v, (uint32_t)row);
+              kb = kq > kb ? kq : kb;
+              if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = v;
+            } break;
+            default: break;
+          }
+        }
+        if (KIND == PH_LM && last_seg && kb) atomicMax(&sm.best[b], kb);
+      }
+      unit_cyc += clock64() - tu;
+      ++unit_cnt;
+    }
+    if (++stage == (uint32_t)n_stages) {
+      stage = 0;
+      phase_bit ^= 1u;
+    }
+  }
+  if (KIND == PH_LM && last_seg) {
+    named_bar_sync(1, kNCT);
+    if (tid_c < B) p.cand[cta * B + tid_c] = sm.best[tid_c];
+  }
+}
+
 template <int B>
 __device__ __forceinline__ void gemv_phase(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                            int k, int s, int tid_c, uint32_t& stage,
@@ -896,6 +1134,25 @@ __device__ __forceinline__ void gemv_phase(const DecodeParams& p, const Smem& sm
                                            long long& unit_cyc, long long& unit_cnt) {
   constexpr int NR = RowsPerUnit<B>::value;
   constexpr int NRG = NR < 2 ? 2 : NR;   // GU units always hold gate/up pairs
+  if constexpr (B >= kTcMinBatch) {
+    switch (ph.kind) {
+      case PH_QKV:
+        gemv_phase_tc<B, PH_QKV>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
+        break;
+      case PH_O:
+        gemv_phase_tc<B, PH_O>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
+        break;
+      case PH_GU:
+        gemv_phase_tc<B, PH_GU>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
+        break;
+      case PH_DOWN:
+        gemv_phase_tc<B, PH_DOWN>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
+        break;
+      default:
+        gemv_phase_tc<B, PH_LM>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
+        break;
+    }
+  } else {
   switch (ph.kind) {
     case PH_QKV:
       gemv_phase_nr<B, NR, PH_QKV>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
@@ -912,6 +1169,7 @@ __device__ __forceinline__ void gemv_phase(const DecodeParams& p, const Smem& sm
     default:
       gemv_phase_nr<B, NR, PH_LM>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, wait_cyc, unit_cyc, unit_cnt);
       break;
+  }
   }
 }
 
@@ -930,6 +1188,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     if (blockIdx.x == 0) p.stamps[0] = globaltimer();
   }
   for (int i = threadIdx.x; i < n_stages * kMaxUnits; i += blockDim.x) sm.cnt[i] = 0;
+  if (B >= kTcMinBatch && threadIdx.x < 16) reinterpret_cast<uint32_t*>(sm.zero)[threadIdx.x] = 0u;
   __syncthreads();
 
   if (warp_id == 0) {

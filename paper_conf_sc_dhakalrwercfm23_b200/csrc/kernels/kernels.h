@@ -34,6 +34,10 @@ constexpr int kXinSegBytes = 64 * 1024; // activation staging per K segment (B *
 #define MX_HD
 #endif
 MX_HD constexpr int decode_seg_cols(int B) { return (kXinSegBytes / (B * 4)) & ~255; }
+// Batch sizes >= kTcMinBatch run the GEMVs on the tensor cores (K7): tiles of
+// 8 weight rows x <= kTcCols columns (one 32 KiB stage with a 16-byte row pad).
+constexpr int kTcMinBatch = 4;
+constexpr int kTcCols = 2016;
 // Activation staging columns for the widest phase input kmax.
 MX_HD constexpr int decode_xin_cols(int B, int kmax) {
   return ((kmax + 255) & ~255) < decode_seg_cols(B) ? ((kmax + 255) & ~255) : decode_seg_cols(B);
@@ -86,6 +90,13 @@ uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 
 // Shared-memory bytes of the decode kernel for a given shape.
 int decode_smem_bytes(int B, int kmax, int* n_stages);
+// Bytes of the activation staging buffer (CUDA-core: fp32 [B][cols]; tensor
+// cores: bf16 hi and lo [B][cols + 8] plus a 64-byte zero block).
+MX_HD constexpr int decode_xin_bytes(int B, int kmax) {
+  return B >= kTcMinBatch
+             ? 2 * B * ((((kmax + 31) & ~31) < kTcCols ? ((kmax + 31) & ~31) : kTcCols) * 2 + 16) + 64
+             : B * decode_xin_cols(B, kmax) * 4;
+}
 
 // cooperative != 0: cuLaunchCooperativeKernel (all CTAs co-resident; used on
 // unpartitioned streams where other kernels compete for the same SMs).

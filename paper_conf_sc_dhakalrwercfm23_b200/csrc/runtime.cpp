@@ -282,9 +282,40 @@ static int make_shared_exec(Gpu& gpu, int n_ctas, uint32_t epoch, std::unique_pt
   return MX_OK;
 }
 
+static uint64_t exec_key(const std::vector<int>& groups, bool whole) {
+  uint64_t m = whole ? (1ull << 63) : 0ull;
+  for (int g : groups) m |= 1ull << g;
+  return m;
+}
+
+// Return an idle green-context exec to the GPU's pool (shared execs are destroyed).
+static void release_exec(Gpu& gpu, std::unique_ptr<Exec> e) {
+  if (!e) return;
+  if (e->shared || !e->gctx) {
+    destroy_exec(e.get());
+    return;
+  }
+  std::lock_guard<std::mutex> lk(gpu.pool_mu);
+  const uint64_t k = e->key;
+  gpu.exec_pool.emplace(k, std::move(e));
+}
+
 static int make_exec(Gpu& gpu, const std::vector<int>& groups, bool whole, uint32_t epoch,
                      std::unique_ptr<Exec>* out) {
+  const uint64_t key = exec_key(groups, whole);
+  {
+    std::lock_guard<std::mutex> lk(gpu.pool_mu);
+    auto it = gpu.exec_pool.find(key);
+    if (it != gpu.exec_pool.end()) {
+      *out = std::move(it->second);
+      gpu.exec_pool.erase(it);
+      (*out)->epoch = epoch;
+      (*out)->inflight = 0;
+      return MX_OK;
+    }
+  }
   auto e = std::make_unique<Exec>();
+  e->key = key;
   e->epoch = epoch;
   CUdevResourceDesc desc;
   if (whole) {
@@ -821,7 +852,7 @@ static void dispatcher_main(Lib* L, Gpu* gpu) {
         }
         for (size_t i = 0; i < p->draining.size();) {
           if (p->draining[i]->inflight == 0) {
-            destroy_exec(p->draining[i].get());
+            release_exec(*gpu, std::move(p->draining[i]));
             p->draining.erase(p->draining.begin() + i);
           } else {
             ++i;
@@ -1061,6 +1092,14 @@ mx_status mx_shutdown(void) {
     destroy_exec(p->cur.get());
     p->arena.release();
   }
+  for (auto& g : L->gpus) {
+    CtxGuard cg(g->primary);
+    for (auto& kv : g->exec_pool) {
+      drv().cuStreamSynchronize(kv.second->stream);
+      destroy_exec(kv.second.get());
+    }
+    g->exec_pool.clear();
+  }
   for (auto& g : L->gpus) drv().cuDevicePrimaryCtxRelease(g->dev);
   g_lib = nullptr;
   delete L;
@@ -1288,8 +1327,7 @@ mx_status part_destroy(int32_t part) {
       if (s.h_stamps) drv().cuMemFreeHost(s.h_stamps);
     }
   p.insts.clear();
-  destroy_exec(p.cur.get());
-  p.cur.reset();
+  release_exec(g, std::move(p.cur));
   p.arena.release();
   p.live = false;
   return L->sched->destroy(part);

@@ -40,6 +40,7 @@ struct Exec {
   uint32_t epoch = 0;
   CUevent ev[2][3] = {};   // per in-flight lane: kernel start, kernel end, done
   int inflight = 0;
+  uint64_t key = 0;        // SM-group mask | whole << 63 (green-context pool key)
 };
 
 struct Task {
@@ -147,6 +148,11 @@ struct Gpu {
   std::condition_variable cv;
   bool stop = false;
   std::vector<Partition*> parts;
+  // Idle green contexts (+ stream + events) by SM-group set. Creating a green
+  // context takes 1-200 ms on a busy device (measured), so part_resize and
+  // part_destroy return execs here and make_exec reuses them.
+  std::mutex pool_mu;
+  std::multimap<uint64_t, std::unique_ptr<Exec>> exec_pool;
 };
 
 }  // namespace mx

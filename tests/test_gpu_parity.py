@@ -69,6 +69,21 @@ def test_ragged_gqa_batch3(mxlib, parts):
     _check_decode(cfg, w, prompt, 9, t.tokens, t.logits)
 
 
+@pytest.mark.parametrize("cfg,B,sm", [(RAGGED, 5, 12), (TINY, 4, 8), (RAGGED, 8, 40)])
+def test_tensor_core_batches(mxlib, parts, cfg, B, sm):
+    """Batch >= 4 runs the GEMVs on the tensor cores (K7, bf16 hi/lo activations):
+    ragged K (264 -> padded 288, masked), ragged rows, GQA, B = 4 / 5 / 8."""
+    p = parts(sm)
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=B))
+    w = decode_weights(cfg)
+    prompt = prompt_tokens(40 + B, B, 6, cfg.vocab)
+    t = mxlib.decode_task(fn, prompt, 7, want_logits=True, vocab=cfg.vocab)
+    mxlib.fn_submit(p, t)
+    assert mxlib.fn_wait(t)["status"] == 0
+    rel = _check_decode(cfg, w, prompt, 7, t.tokens, t.logits)
+    print(f"TC {cfg.name} B={B}: max rel err {rel:.2e}")
+
+
 def test_single_token_generation_and_single_prompt(mxlib, parts):
     """Degenerate shapes: G = 1 (one LM-head step) and P = 1 (no prompt steps)."""
     cfg = TINY

@@ -13,6 +13,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_sc_dhakalrwercfm23_b200 import mx  # noqa: E402
 from workloads.configs import DECODE_CFGS  # noqa: E402
 from workloads.inputs import prompt_tokens  # noqa: E402
+from paper_conf_sc_dhakalrwercfm23_b200.metrics import decode_task_bytes  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--sms", type=int, default=12)
@@ -42,7 +43,6 @@ for k in range(a.tasks):
     h0 = time.perf_counter()
     mx.fn_submit(p, t)
     r = mx.fn_wait(t)
-    from oracle.cost import decode_task_bytes
     gbs = decode_task_bytes(cfg, a.batch, a.P, a.G) / r['kernel_ns']
     print(f"task {k}: status {r['status']} kernel {r['kernel_ns'] / 1e6:.3f} ms  {gbs:.1f} GB/s "
           f"({gbs / mx.part_query(p)['n_ctas']:.1f} GB/s/SM) "
