@@ -258,6 +258,24 @@ mx_status mx_sched_submit(mx_sched* s, int32_t fn, int32_t part, uint64_t cost,
 /* Serialise the canonical trace into buf (cap bytes); *len = bytes needed. */
 mx_status mx_sched_trace(const mx_sched* s, void* buf, uint64_t cap, uint64_t* len);
 
+/* ---------------------------------------------------------------------------
+ * Right-sizing policy (Fig. 2
+ * "LLaMa2 can only properly utilize about 20 SMs", future work P:252). Host
+ * only. Input: a function's single-instance service time t[i] (any time unit)
+ * measured alone on sms[i] SMs (the D2b sweep; n_points >= 1, sms ascending,
+ * each > 0). Output: a partition size *out_sm (one of sms[]) and a count
+ * *out_parts of equal partitions for a device of total_sms SMs (<= max_parts),
+ * with the predicted throughput *out_rate = parts / t (tasks per time unit):
+ *   objective 0 (latency knee): the smallest sms[i] with
+ *                t[i] <= (1 + slack) * min_j t[j];
+ *   objective 1 (throughput):   argmax_i floor(total_sms / sms[i]) / t[i]
+ *                (exact ties -> the larger partition, i.e. lower latency).
+ * Errors: MX_EINVAL on null pointers, n_points < 1, non-positive or
+ * non-ascending sms, non-positive t, slack < 0, or no size fitting total_sms. */
+mx_status mx_rightsize(const int32_t* sms, const double* t, int32_t n_points, int32_t total_sms,
+                       int32_t max_parts, int32_t objective, double slack, int32_t* out_sm,
+                       int32_t* out_parts, double* out_rate);
+
 #ifdef __cplusplus
 }
 #endif

@@ -1691,4 +1691,39 @@ mx_status mx_sched_trace(const mx_sched* s, void* buf, uint64_t cap, uint64_t* l
   return MX_OK;
 }
 
+mx_status mx_rightsize(const int32_t* sms, const double* t, int32_t n_points, int32_t total_sms,
+                       int32_t max_parts, int32_t objective, double slack, int32_t* out_sm,
+                       int32_t* out_parts, double* out_rate) {
+  if (!sms || !t || !out_sm || !out_parts || n_points < 1 || total_sms < 1 || max_parts < 1 ||
+      !(slack >= 0.0) || (objective != 0 && objective != 1))
+    return MX_EINVAL;
+  double tmin = 0.0;
+  for (int i = 0; i < n_points; ++i) {
+    if (sms[i] <= 0 || !(t[i] > 0.0) || (i > 0 && sms[i] <= sms[i - 1])) return MX_EINVAL;
+    if (i == 0 || t[i] < tmin) tmin = t[i];
+  }
+  int best = -1;
+  int best_parts = 0;
+  for (int i = 0; i < n_points; ++i) {
+    if (sms[i] > total_sms) break;
+    const int parts = std::min(max_parts, total_sms / sms[i]);
+    if (objective == 0) {
+      if (t[i] <= (1.0 + slack) * tmin) {
+        best = i;
+        best_parts = parts;
+        break;
+      }
+    } else if (best < 0 || (double)parts * t[best] >= (double)best_parts * t[i]) {
+      // parts / t[i] >= best_parts / t[best]; ascending sms -> ties go to the larger size
+      best = i;
+      best_parts = parts;
+    }
+  }
+  if (best < 0) return MX_EINVAL;
+  *out_sm = sms[best];
+  *out_parts = best_parts;
+  if (out_rate) *out_rate = (double)best_parts / t[best];
+  return MX_OK;
+}
+
 }  // extern "C"

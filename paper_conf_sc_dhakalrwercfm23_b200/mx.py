@@ -112,6 +112,9 @@ _SIGS = {
     "mx_sched_submit": (C.c_int32, [C.c_void_p, C.c_int32, C.c_int32, C.c_uint64,
                                     C.POINTER(C.c_uint64), C.POINTER(C.c_int32),
                                     C.POINTER(C.c_uint64)]),
+    "mx_rightsize": (C.c_int32, [C.POINTER(C.c_int32), C.POINTER(C.c_double), C.c_int32, C.c_int32,
+                                 C.c_int32, C.c_int32, C.c_double, C.POINTER(C.c_int32),
+                                 C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
     "mx_sched_trace": (C.c_int32, [C.c_void_p, C.c_void_p, C.c_uint64, C.POINTER(C.c_uint64)]),
 }
 
@@ -344,6 +347,17 @@ def launch_count() -> int:
     c = C.c_uint64()
     _check(lib().mx_launch_count(C.byref(c)), "mx_launch_count")
     return c.value
+
+
+def rightsize(sms, t, total_sms=148, max_parts=37, objective=1, slack=0.0):
+    """N2 right-sizing (mx_rightsize): -> (sm_per_partition, n_partitions, predicted rate)."""
+    n = len(sms)
+    a = (C.c_int32 * n)(*[int(x) for x in sms])
+    b = (C.c_double * n)(*[float(x) for x in t])
+    o_sm, o_p, o_r = C.c_int32(), C.c_int32(), C.c_double()
+    _check(lib().mx_rightsize(a, b, n, total_sms, max_parts, objective, slack, C.byref(o_sm),
+                              C.byref(o_p), C.byref(o_r)), "mx_rightsize")
+    return o_sm.value, o_p.value, o_r.value
 
 
 # ---------------------------------------------------------------------------

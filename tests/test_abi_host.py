@@ -118,3 +118,30 @@ def test_task_validation_rejects_bad_inputs():
     over = mx.decode_desc(LLAMA7B, max_batch=9)  # batch > 8
     with pytest.raises(mx.MxError):
         mx.task_default_cost(over, mx.decode_task(1, np.zeros((9, 4), dtype=np.int32), 4))
+
+
+def test_rightsize_policy_n2():
+    """N2 right-sizing (mx_rightsize), pinned on hand-computed cases: the
+    throughput objective maximises floor(148/s)/t(s); the latency objective
+    takes the smallest size within (1+slack) of the fastest; ties and the
+    max_parts cap; invalid inputs."""
+    # D2b-shaped curve (GPT-2s decode, ms per task alone on s SMs)
+    sms = [4, 8, 12, 16, 24, 32, 48, 64, 72, 96, 120, 148]
+    t = [62.1, 38.9, 31.7, 27.3, 23.9, 22.1, 20.0, 19.8, 19.5, 19.3, 18.8, 18.96]
+    s, n, rate = mx.rightsize(sms, t, objective=1)
+    assert (s, n) == (4, 37) and abs(rate - 37 / 62.1) < 1e-12
+    s, n, _ = mx.rightsize(sms, t, objective=0, slack=0.10)   # <= 20.68 ms
+    assert (s, n) == (48, 3)
+    s, n, _ = mx.rightsize(sms, t, objective=0, slack=0.0)    # the fastest point
+    assert (s, n) == (120, 1)
+    # efficiency peaking in the middle: 37/100, 18/30, 9/20 -> 8 SMs
+    assert mx.rightsize([4, 8, 16], [100.0, 30.0, 20.0])[:2] == (8, 18)
+    # exact tie 2/2 == 1/1 -> the larger partition
+    assert mx.rightsize([4, 8], [2.0, 1.0], total_sms=8)[:2] == (8, 1)
+    # max_parts caps the count: 2/1 vs 2/1.5 -> 4 SMs x 2
+    assert mx.rightsize([4, 8], [1.0, 1.5], max_parts=2)[:2] == (4, 2)
+    for bad in (dict(sms=[8, 4], t=[1.0, 1.0]), dict(sms=[4], t=[0.0]),
+                dict(sms=[200], t=[1.0]), dict(sms=[4], t=[1.0], slack=-1.0, objective=0)):
+        with pytest.raises(mx.MxError) as e:
+            mx.rightsize(**bad)
+        assert e.value.code == mx.MX_EINVAL
