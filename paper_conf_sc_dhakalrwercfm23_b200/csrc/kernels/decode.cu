@@ -27,6 +27,14 @@ int decode_smem_bytes(int B, int kmax, int* n_stages) {
 
 // Fused (per-CTA) attention only for small attention on the CUDA-core path
 // (the tensor-core path stages its activations as bf16 hi/lo, not fp32).
+int decode_prof_buckets() {
+#ifdef MX_PROF_BUCKETS
+  return 1;
+#else
+  return 0;
+#endif
+}
+
 int decode_fuse_attention(int B, int H, int hd) {
   return (B < kTcMinBatch && B * H * hd <= 1024) ? 1 : 0;
 }

@@ -64,6 +64,15 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
   }
 }
 
+// Per-CTA cycle buckets (MX_DECODE_PROF=1) exist only in profiling builds
+// (MX_DEFS=-DMX_PROF_BUCKETS): in the product build the counters fold to
+// constants and cost no registers in the GEMV loop.
+#ifdef MX_PROF_BUCKETS
+#define MX_CLK() clock64()
+#else
+#define MX_CLK() 0ll
+#endif
+
 constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
 
 // One GEMV phase, or one K segment of it. Phases whose staged activations
@@ -295,9 +304,9 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
           const int n = min(ph.TR, r1 - r);
           // never abandons the stream: after a barrier timeout the consumers run
           // through the remaining phases without waiting, so every slot is freed.
-          const long long tw = clock64();
+          const long long tw = MX_CLK();
           mbar_wait_bounded(&sm.empty[stage], phase_bit ^ 1u, p.err);
-          wait_cyc += clock64() - tw;
+          wait_cyc += MX_CLK() - tw;
           const uint32_t one = (uint32_t)n * (uint32_t)ph.K * 2u;
           const uint32_t total = (kind == PH_GU) ? 2u * one : one;
           uint8_t* dst = sm.ring + (size_t)stage * kStageBytes;
@@ -816,14 +825,14 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
     start = (start + units) % kConsumerWarps;
     // every warp observes the stage fill before releasing it (keeps the empty
     // barrier's arrival count per round exact)
-    const long long tw = clock64();
+    const long long tw = MX_CLK();
     mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
-    wait_cyc += clock64() - tw;
+    wait_cyc += MX_CLK() - tw;
     const uint16_t* wt = reinterpret_cast<const uint16_t*>(sm.ring + (size_t)stage * kStageBytes);
     float* red = sm.red + (size_t)stage * kMaxUnits * B;
     int* cnt = sm.cnt + stage * kMaxUnits;
     for (; u < units; u += kConsumerWarps) {
-      const long long tu = clock64();
+      const long long tu = MX_CLK();
       const int gi = (NG == 1) ? u : u / NG;   // output group within the tile
       const int g = u - gi * NG;
       const int j0 = gi * per;                 // first tile-local output of the unit
@@ -946,7 +955,7 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
           default: break;
         }
       }
-      unit_cyc += clock64() - tu;
+      unit_cyc += MX_CLK() - tu;
       ++unit_cnt;
     }
     __syncwarp();
@@ -1008,9 +1017,9 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
     // (count kConsumerWarps): a parity wait only tells two consecutive phases
     // apart, so no warp may skip stages and run a full ring ahead. Only the
     // owner warp computes the tile.
-    const long long tw = clock64();
+    const long long tw = MX_CLK();
     mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
-    const long long tu = clock64();
+    const long long tu = MX_CLK();
     wait_cyc += tu - tw;
     if (gidx % kConsumerWarps != warp) {
       __syncwarp();
@@ -1113,7 +1122,7 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
         }
         if (KIND == PH_LM && last_seg && kb) atomicMax(&sm.best[b], kb);
       }
-      unit_cyc += clock64() - tu;
+      unit_cyc += MX_CLK() - tu;
       ++unit_cnt;
     }
     if (++stage == (uint32_t)n_stages) {
@@ -1202,16 +1211,16 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
   uint32_t stage = 0, phase_bit = 0;
   unsigned long long target = p.bar_base;
   long long c_bar = 0, c_stage = 0, c_wait = 0, c_gemv = 0, c_att = 0, c_unit = 0, c_units = 0;
-  const long long t_begin = clock64();
+  const long long t_begin = MX_CLK();
   for (int s = 0; s < S; ++s) {
     const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
     for (int k = 0; k < nph; ++k) {
       const int kind = phase_kind(k, L, p.fuse_att);
       const int layer = k / pl;
-      long long t0 = clock64();
+      long long t0 = MX_CLK();
       if (kind == PH_ATT) {
         attention_phase<B>(p, sm, layer, s, tid_c);
-        const long long t1 = clock64();
+        const long long t1 = MX_CLK();
         c_att += t1 - t0;
         t0 = t1;
       } else {
@@ -1219,25 +1228,25 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         for (int seg = 0; seg < nseg; ++seg) {
           const Phase ph = make_phase<B>(p, kind, layer, seg);
           stage_input<B>(p, sm, ph, s, tid_c);
-          const long long t1 = clock64();
+          const long long t1 = MX_CLK();
           if (kind == PH_O && p.fuse_att)
             c_att += t1 - t0;
           else
             c_stage += t1 - t0;
           gemv_phase<B>(p, sm, ph, k, s, tid_c, stage, phase_bit, n_stages, c_wait, c_unit, c_units);
-          const long long t2 = clock64();
+          const long long t2 = MX_CLK();
           c_gemv += t2 - t1;
           t0 = t2;
         }
       }
       target += (unsigned long long)p.n_ctas;
       grid_barrier(p, target, tid_c);
-      c_bar += clock64() - t0;
+      c_bar += MX_CLK() - t0;
     }
   }
   if (p.prof && tid_c == 0) {
     unsigned long long* pr = p.prof + blockIdx.x * 16;
-    pr[0] = (unsigned long long)(clock64() - t_begin);
+    pr[0] = (unsigned long long)(MX_CLK() - t_begin);
     pr[1] = (unsigned long long)c_bar;
     pr[2] = (unsigned long long)c_stage;
     pr[3] = (unsigned long long)c_wait;

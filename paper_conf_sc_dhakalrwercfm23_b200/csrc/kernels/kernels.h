@@ -85,6 +85,8 @@ struct DecodeParams {
 
 // 1 if every CTA computes the whole attention itself (B*H*hd <= 1024).
 int decode_fuse_attention(int B, int H, int hd);
+// 1 if this build records the per-CTA cycle buckets (-DMX_PROF_BUCKETS).
+int decode_prof_buckets();
 // Number of grid barriers one decode launch performs (host bookkeeping of bar_base).
 uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 

@@ -977,6 +977,9 @@ static int init_impl(const std::vector<int>& ordinals) {
   setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
   g_decode_prof = getenv("MX_DECODE_PROF") && atoi(getenv("MX_DECODE_PROF")) == 1;
   g_trace_resize = getenv("MX_TRACE_RESIZE") && atoi(getenv("MX_TRACE_RESIZE")) == 1;
+  if (g_decode_prof && !mxk::decode_prof_buckets())
+    fprintf(stderr, "[mx] MX_DECODE_PROF=1 needs a build with MX_DEFS=-DMX_PROF_BUCKETS; "
+                    "the cycle buckets will read 0\n");
   if (const char* e = getenv("MX_INFLIGHT")) {
     const int v = atoi(e);
     g_inflight_override = (v == 1 || v == 2) ? (size_t)v : 0;
