@@ -73,7 +73,10 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
 #define MX_CLK() 0ll
 #endif
 
-constexpr int kCPG = 8;                     // 256-column chunks per GEMV work unit
+#ifndef MX_CPG
+#define MX_CPG 8
+#endif
+constexpr int kCPG = MX_CPG;                // 256-column chunks per GEMV work unit
 
 // One GEMV phase, or one K segment of it. Phases whose staged activations
 // (B * K * 4 bytes) exceed kXinSegBytes run as `nseg` column segments

@@ -7,16 +7,23 @@
 // Computed as h' = ReLU(c + U h + sum_b W_b s_b) with s_b[v] = sum over
 // type-b bonds of v of the neighbour's h (linearity; reading R7).
 //
-// B200 design: the per-step transforms are dense [atoms x 128] x [128 x 128]
-// contractions, so they run on the tensor cores. Molecules are packed (host,
-// deterministic greedy) into tiles of <= 128 atoms; a CTA (8 warps) owns a
-// tile, warp w owns atom rows 16w..16w+15 and all 128 output features
-// (64 fp32 accumulators per thread). Activations are fed as a bf16 hi/lo pair
-// (x = hi + lo, two MMAs: ~16-bit mantissa, reading A17), weights are exact in
-// bf16. Operands sit in shared memory with a 16-byte XOR swizzle and are
-// fetched with ldmatrix; the next weight matrix is prefetched with cp.async
-// while the current one is consumed. mma.sync m16n8k16 (legacy tensor path)
-// in round 1; tcgen05/TMEM is NEXT.
+// B200 design: the per-step transforms are dense [128 atoms x 128] x [128 x 128]
+// contractions, so they run on the 5th-generation tensor cores (tcgen05).
+// Molecules are packed (host, deterministic greedy) into tiles of <= 128
+// atoms; a CTA (8 warps) owns a tile. Per message-passing step the five
+// contractions U.h, W_0.s_0 .. W_3.s_3 accumulate into ONE 128 x 128 fp32
+// accumulator in tensor memory (TMEM, 128 columns): one elected thread issues
+// tcgen05.mma (M=128, N=128, K=16, bf16 x bf16 -> fp32) straight from shared
+// memory descriptors and commits to an mbarrier. Activations are fed as a bf16
+// hi/lo pair (x = hi + lo, two MMAs: ~16-bit mantissa, reading A17); weights
+// are exact in bf16. Operands sit in shared memory in the canonical UMMA
+// K-major SWIZZLE_128B layout (each [128][128] operand = two [128][64] halves
+// of 8-row x 128-byte swizzle atoms). While the U.h contraction runs on the
+// tensor cores, the CUDA cores build the first neighbour sum s_b; the next
+// weight matrix is prefetched with cp.async while the current one is consumed.
+// The epilogue reads the accumulator with tcgen05.ld (warp w owns TMEM lanes
+// 32(w%4).. and half the columns), applies +c and ReLU and writes the next h
+// (hi/lo) back into the swizzled operand.
 #include "common.cuh"
 #include "kernels.h"
 #include "launch.cuh"
@@ -27,9 +34,11 @@ constexpr int kF = 128;
 constexpr int kTileAtoms = 128;
 constexpr int kTileEdges = 512;
 constexpr int kMpnnThreads = 256;
-constexpr int kMatBytes = kF * kF * 2;        // one 128x128 bf16 operand
+constexpr int kMatBytes = kF * kF * 2;        // one 128x128 bf16 operand (two 16 KiB halves)
+constexpr int kHalfBytes = kMatBytes / 2;     // [128 rows][64 cols] SWIZZLE_128B region
+constexpr int kTmemCols = 128;                // fp32 accumulator 128 lanes x 128 columns
 
-// smem map
+// smem map (offsets from a 1024-byte aligned base)
 constexpr int kOffHhi = 0;
 constexpr int kOffHlo = kOffHhi + kMatBytes;
 constexpr int kOffShi = kOffHlo + kMatBytes;
@@ -42,14 +51,23 @@ constexpr int kOffNbrOff = kOffMolE + kTileAtoms * 8;          // int [kTileAtom
 constexpr int kOffNbr = kOffNbrOff + (kTileAtoms + 4) * 4;     // int [2*kTileEdges]: (u<<2)|b
 constexpr int kReadoutMols = 4;                                // molecules per readout batch
 constexpr int kOffR = kOffNbr + 2 * kTileEdges * 4;            // float [kReadoutMols][2][kF]: r, z
-constexpr int kOffRed = kOffR + kReadoutMols * 2 * kF * 4;     // float [16]
-constexpr int kMpnnSmem = kOffRed + 64;
+constexpr int kOffC = kOffR + kReadoutMols * 2 * kF * 4;       // float [kF]: bias c
+constexpr int kOffRed = kOffC + kF * 4;                        // float [16]
+constexpr int kOffBar = kOffRed + 64;                          // uint64 mbarrier (MMA done)
+constexpr int kOffTmem = kOffBar + 8;                          // uint32 TMEM base address
+constexpr int kMpnnSmem = kOffTmem + 8 + 1024;                 // + alignment slack
 
 int mpnn_smem_bytes() { return kMpnnSmem; }
 
-// byte offset of element (row, col) of a swizzled [128][128] bf16 operand
-__device__ __forceinline__ uint32_t sw_off(int row, int col) {
-  return (uint32_t)(row * 256 + ((((col >> 3) ^ (row & 7))) << 4) + (col & 7) * 2);
+// Byte offset of 16-byte chunk `ch` (columns 8ch..8ch+7) of row `row` in a
+// [128][128] bf16 operand stored as two K-major SWIZZLE_128B halves: half
+// ch>>3 holds columns 64*(ch>>3).., rows are 128 bytes, 8-row atoms of 1024
+// bytes, chunk index XOR (row & 7) inside an atom.
+__device__ __forceinline__ uint32_t chunk_off(int row, int ch) {
+  return (uint32_t)((ch >> 3) * kHalfBytes + row * 128 + ((((ch & 7) ^ (row & 7))) << 4));
+}
+__device__ __forceinline__ uint32_t elem_off(int row, int col) {
+  return chunk_off(row, col >> 3) + (col & 7) * 2;
 }
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
@@ -57,12 +75,67 @@ __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+// generic-proxy smem writes (st.shared, cp.async) -> visible to the tensor core (async proxy)
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+
+// UMMA shared-memory descriptor, K-major SWIZZLE_128B: start address >> 4
+// (bits 0-13), leading byte offset (unused for swizzled K-major, 16 B) >> 4
+// (16-29), stride byte offset = 1024 B between 8-row atoms >> 4 (32-45),
+// descriptor version 1 (46-47), layout type SWIZZLE_128B = 2 (61-63).
+__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
+  return (uint64_t)((saddr >> 4) & 0x3FFF) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+
+// Instruction descriptor, kind::f16: D fp32 (bits 4-5 = 1), A bf16 (7-9 = 1),
+// B bf16 (10-12 = 1), A and B K-major (15, 16 = 0), N >> 3 (17-22), M >> 4 (24-28).
+constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kF >> 3) << 17) |
+                            ((uint32_t)(kTileAtoms >> 4) << 24);
+
+__device__ __forceinline__ void umma_bf16(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(kIdesc), "r"(accumulate)
+      : "memory");
+}
+
+__device__ __forceinline__ void umma_commit(uint32_t bar_saddr) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   bar_saddr)
+               : "memory");
+}
+
+// 16 consecutive fp32 accumulator columns of this thread's TMEM lane.
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, "
+      "%12, %13, %14, %15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
 
 // Async load of a row-major [128][128] bf16 matrix (global) into a swizzled smem operand.
 __device__ __forceinline__ void load_matrix_async(uint32_t dst_base, const uint16_t* src, int tid) {
   for (int i = tid; i < kF * kF / 8; i += kMpnnThreads) {
     const int row = i >> 4, ch = i & 15;
-    cp_async16(dst_base + (uint32_t)(row * 256 + ((ch ^ (row & 7)) << 4)), src + (size_t)i * 8);
+    cp_async16(dst_base + chunk_off(row, ch), src + (size_t)i * 8);
   }
   cp_async_commit();
 }
@@ -73,47 +146,87 @@ __device__ __forceinline__ void split_bf16(float x, uint16_t& hi, uint16_t& lo) 
   lo = f32_to_bf16_rne(x - bf16_bits_to_f32(hi));
 }
 
-// acc[16 n-tiles][4] += A(16 rows of this warp, 128 k) . W^T  for A given as hi+lo.
-__device__ __forceinline__ void mma_segment(float (&acc)[16][4], uint32_t a_hi, uint32_t a_lo,
-                                            uint32_t w, int warp, int lane) {
-  const int q = lane >> 3, r = lane & 7;
-  const int arow = warp * 16 + (q & 1) * 8 + r;
-#pragma unroll 2
-  for (int k0 = 0; k0 < kF; k0 += 16) {
-    const int acol = k0 + (q >> 1) * 8;
-    uint32_t h0, h1, h2, h3, l0, l1, l2, l3;
-    ldsm_x4(a_hi + sw_off(arow, acol), h0, h1, h2, h3);
-    ldsm_x4(a_lo + sw_off(arow, acol), l0, l1, l2, l3);
+__device__ __forceinline__ void split_store8(uint8_t* hi_dst, uint8_t* lo_dst, const float (&v)[8]) {
+  uint16_t sh[8], sl[8];
 #pragma unroll
-    for (int nt = 0; nt < 16; nt += 2) {
-      const int brow = nt * 8 + r + (q >> 1) * 8;
-      const int bcol = k0 + (q & 1) * 8;
-      uint32_t b0, b1, b2, b3;
-      ldsm_x4(w + sw_off(brow, bcol), b0, b1, b2, b3);
-      mma_bf16(acc[nt], h0, h1, h2, h3, b0, b1);
-      mma_bf16(acc[nt], l0, l1, l2, l3, b0, b1);
-      mma_bf16(acc[nt + 1], h0, h1, h2, h3, b2, b3);
-      mma_bf16(acc[nt + 1], l0, l1, l2, l3, b2, b3);
+  for (int j = 0; j < 8; ++j) split_bf16(v[j], sh[j], sl[j]);
+  uint4 ph, pl;
+  ph.x = sh[0] | ((uint32_t)sh[1] << 16); ph.y = sh[2] | ((uint32_t)sh[3] << 16);
+  ph.z = sh[4] | ((uint32_t)sh[5] << 16); ph.w = sh[6] | ((uint32_t)sh[7] << 16);
+  pl.x = sl[0] | ((uint32_t)sl[1] << 16); pl.y = sl[2] | ((uint32_t)sl[3] << 16);
+  pl.z = sl[4] | ((uint32_t)sl[5] << 16); pl.w = sl[6] | ((uint32_t)sl[7] << 16);
+  *reinterpret_cast<uint4*>(hi_dst) = ph;
+  *reinterpret_cast<uint4*>(lo_dst) = pl;
+}
+
+// s_b[v] = sum over type-b bonds of v of h[neighbour] (neighbour-list order),
+// written as a hi/lo operand; padded rows are 0.
+__device__ __forceinline__ void build_s(uint8_t* sm, const int* nbr_off, const int* nbr, int na,
+                                        int b, int tid) {
+  for (int i = tid; i < kTileAtoms * 16; i += kMpnnThreads) {
+    const int v = i >> 4, ch = i & 15;
+    float sacc[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) sacc[j] = 0.f;
+    if (v < na) {
+      for (int q = nbr_off[v]; q < nbr_off[v + 1]; ++q) {
+        const int nb = nbr[q];
+        if ((nb & 3) != b) continue;
+        const uint32_t off = chunk_off(nb >> 2, ch);
+        const uint4 hh = *reinterpret_cast<const uint4*>(sm + kOffHhi + off);
+        const uint4 hl = *reinterpret_cast<const uint4*>(sm + kOffHlo + off);
+        float fh[8], fl[8];
+        unpack8(hh, fh);
+        unpack8(hl, fl);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) sacc[j] += fh[j] + fl[j];
+      }
     }
+    const uint32_t off = chunk_off(v, ch);
+    split_store8(sm + kOffShi + off, sm + kOffSlo + off, sacc);
   }
 }
 
 __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
-  extern __shared__ __align__(1024) uint8_t smem_raw[];
-  const uint32_t sbase = smem_u32(smem_raw);
+  extern __shared__ __align__(1024) uint8_t smem_dyn[];
+  // UMMA SWIZZLE_128B operands need 1024-byte aligned atoms
+  uint8_t* sm = smem_dyn + ((1024 - (smem_u32(smem_dyn) & 1023)) & 1023);
+  const uint32_t sbase = smem_u32(sm);
   const uint32_t Hhi = sbase + kOffHhi, Hlo = sbase + kOffHlo;
   const uint32_t Shi = sbase + kOffShi, Slo = sbase + kOffSlo;
   const uint32_t Wbuf[2] = {sbase + kOffW0, sbase + kOffW1};
-  int4* ed = reinterpret_cast<int4*>(smem_raw + kOffEdges);
-  int2* mol_e = reinterpret_cast<int2*>(smem_raw + kOffMolE);
-  int* nbr_off = reinterpret_cast<int*>(smem_raw + kOffNbrOff);
-  int* nbr = reinterpret_cast<int*>(smem_raw + kOffNbr);
-  float* rz = reinterpret_cast<float*>(smem_raw + kOffR);
-  float* red = reinterpret_cast<float*>(smem_raw + kOffRed);
+  int4* ed = reinterpret_cast<int4*>(sm + kOffEdges);
+  int2* mol_e = reinterpret_cast<int2*>(sm + kOffMolE);
+  int* nbr_off = reinterpret_cast<int*>(sm + kOffNbrOff);
+  int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
+  float* rz = reinterpret_cast<float*>(sm + kOffR);
+  float* cvec = reinterpret_cast<float*>(sm + kOffC);
+  float* red = reinterpret_cast<float*>(sm + kOffRed);
+  uint64_t* mma_bar = reinterpret_cast<uint64_t*>(sm + kOffBar);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sm + kOffTmem);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int g = lane >> 2, t4 = lane & 3;
   if (blockIdx.x == 0 && tid == 0) p.stamps[0] = globaltimer();
   const uint8_t* eb = reinterpret_cast<const uint8_t*>(p.edges);
+
+  // one-time setup: MMA-completion mbarrier, TMEM accumulator (warp 0 owns alloc/dealloc), bias
+  if (tid == 0) {
+    mbar_init(mma_bar, 1);
+    fence_mbar_init();
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(kTmemCols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  for (int i = tid; i < kF; i += kMpnnThreads) cvec[i] = bf16_bits_to_f32(p.c[i]);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  uint32_t mma_phase = 0;
+  const uint32_t bar_s = smem_u32(mma_bar);
 
   for (int tile = blockIdx.x; tile < p.n_tiles; tile += p.n_ctas) {
     const int m0 = p.tile_off[tile], m1 = p.tile_off[tile + 1];
@@ -150,9 +263,9 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       const int row = i >> 4, ch = i & 15;
       uint4 hv = make_uint4(0, 0, 0, 0);
       if (row < na) hv = *reinterpret_cast<const uint4*>(p.e_atom + (size_t)p.atom_type[a0 + row] * kF + ch * 8);
-      const uint32_t off = (uint32_t)(row * 256 + ((ch ^ (row & 7)) << 4));
-      *reinterpret_cast<uint4*>(smem_raw + kOffHhi + off) = hv;
-      *reinterpret_cast<uint4*>(smem_raw + kOffHlo + off) = make_uint4(0, 0, 0, 0);
+      const uint32_t off = chunk_off(row, ch);
+      *reinterpret_cast<uint4*>(sm + kOffHhi + off) = hv;
+      *reinterpret_cast<uint4*>(sm + kOffHlo + off) = make_uint4(0, 0, 0, 0);
     }
     __syncthreads();
     // per-atom neighbour lists (CSR) in edge order: deterministic, built once per tile
@@ -192,91 +305,78 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
     // which bond types occur in the tile (uniform loop, smem broadcast)
     int present = 0;
     for (int i = 0; i < ne; ++i) present |= 1 << ed[i].z;
+    // segments: 0 = U . h, 1..4 = W_b . s_b for bond types present
+    int seg_list[5];
+    int nseg = 0;
+    seg_list[nseg++] = 0;
+    for (int b = 0; b < p.n_bonds; ++b)
+      if (present & (1 << b)) seg_list[nseg++] = 1 + b;
 
     int wi = 0;   // weight buffer in use
     load_matrix_async(Wbuf[wi], p.u, tid);
     for (int step = 0; step < p.T; ++step) {
-      float acc[16][4];
-#pragma unroll
-      for (int nt = 0; nt < 16; ++nt)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[nt][j] = 0.f;
-      // segments: 0 = U . h, 1..4 = W_b . s_b for bond types present
-      int seg_next[5];
-      int nseg = 0;
-      seg_next[nseg++] = 0;
-      for (int b = 0; b < p.n_bonds; ++b)
-        if (present & (1 << b)) seg_next[nseg++] = 1 + b;
+      bool s_ready = false;
       for (int si = 0; si < nseg; ++si) {
-        const int seg = seg_next[si];
+        const int seg = seg_list[si];
+        if (seg > 0 && !s_ready) build_s(sm, nbr_off, nbr, na, seg - 1, tid);
+        s_ready = false;
+        cp_async_wait_all();
+        fence_proxy_async();                   // S / H / W writes -> tensor-core reads
+        tc_fence_before();
+        __syncthreads();                       // weights + S visible; other W buffer free
         // prefetch the next segment's weights (or U of the next step)
         const uint16_t* nxt = nullptr;
-        if (si + 1 < nseg) nxt = p.w_b + (size_t)(seg_next[si + 1] - 1) * kF * kF;
+        if (si + 1 < nseg) nxt = p.w_b + (size_t)(seg_list[si + 1] - 1) * kF * kF;
         else if (step + 1 < p.T) nxt = p.u;
-        uint32_t a_hi = Hhi, a_lo = Hlo;
-        if (seg > 0) {
-          // s_b[v] = sum over type-b bonds of v of h[neighbour], edge order
-          const int b = seg - 1;
-          for (int i = tid; i < kTileAtoms * 16; i += kMpnnThreads) {
-            const int v = i >> 4, ch = i & 15;
-            float sacc[8];
+        if (tid == 0) {
+          tc_fence_after();
+          const uint32_t a_hi = seg > 0 ? Shi : Hhi, a_lo = seg > 0 ? Slo : Hlo;
+          const uint32_t w = Wbuf[wi];
 #pragma unroll
-            for (int j = 0; j < 8; ++j) sacc[j] = 0.f;
-            if (v < na) {
-              for (int q = nbr_off[v]; q < nbr_off[v + 1]; ++q) {
-                const int nb = nbr[q];
-                if ((nb & 3) != b) continue;
-                const int other = nb >> 2;
-                const uint32_t off = (uint32_t)(other * 256 + ((ch ^ (other & 7)) << 4));
-                const uint4 hh = *reinterpret_cast<const uint4*>(smem_raw + kOffHhi + off);
-                const uint4 hl = *reinterpret_cast<const uint4*>(smem_raw + kOffHlo + off);
-                float fh[8], fl[8];
-                unpack8(hh, fh);
-                unpack8(hl, fl);
-#pragma unroll
-                for (int j = 0; j < 8; ++j) sacc[j] += fh[j] + fl[j];
-              }
-            }
-            uint16_t sh[8], sl[8];
-#pragma unroll
-            for (int j = 0; j < 8; ++j) split_bf16(sacc[j], sh[j], sl[j]);
-            const uint32_t off = (uint32_t)(v * 256 + ((ch ^ (v & 7)) << 4));
-            uint4 ph, pl;
-            ph.x = sh[0] | ((uint32_t)sh[1] << 16); ph.y = sh[2] | ((uint32_t)sh[3] << 16);
-            ph.z = sh[4] | ((uint32_t)sh[5] << 16); ph.w = sh[6] | ((uint32_t)sh[7] << 16);
-            pl.x = sl[0] | ((uint32_t)sl[1] << 16); pl.y = sl[2] | ((uint32_t)sl[3] << 16);
-            pl.z = sl[4] | ((uint32_t)sl[5] << 16); pl.w = sl[6] | ((uint32_t)sl[7] << 16);
-            *reinterpret_cast<uint4*>(smem_raw + kOffShi + off) = ph;
-            *reinterpret_cast<uint4*>(smem_raw + kOffSlo + off) = pl;
+          for (int kk = 0; kk < kF / 16; ++kk) {
+            const uint32_t koff = (uint32_t)((kk >> 2) * kHalfBytes + (kk & 3) * 32);
+            const uint64_t bdesc = umma_desc_sw128(w + koff);
+            umma_bf16(tmem, umma_desc_sw128(a_hi + koff), bdesc, (si > 0 || kk > 0) ? 1u : 0u);
+            umma_bf16(tmem, umma_desc_sw128(a_lo + koff), bdesc, 1u);
           }
-          a_hi = Shi;
-          a_lo = Slo;
+          umma_commit(bar_s);                  // arrives when these MMAs have completed
         }
-        cp_async_wait_all();
-        __syncthreads();                       // weights + S visible; previous W buffer free
         if (nxt) load_matrix_async(Wbuf[wi ^ 1], nxt, tid);
-        mma_segment(acc, a_hi, a_lo, Wbuf[wi], warp, lane);
+        // the U.h contraction does not read S: build the next neighbour sum under it
+        if (seg == 0 && si + 1 < nseg) {
+          build_s(sm, nbr_off, nbr, na, seg_list[si + 1] - 1, tid);
+          s_ready = true;
+        }
+        while (!mbar_try_wait_sleep(mma_bar, mma_phase, 1000)) {
+        }
+        mma_phase ^= 1;
         wi ^= 1;
-        __syncthreads();                       // S / W consumed before they are rewritten
       }
-      // h = ReLU(acc + c) -> hi/lo (padded rows stay 0)
+      // epilogue: h = ReLU(acc + c) -> hi/lo operand (padded rows stay 0).
+      // warp w: TMEM lanes 32(w%4).. (= atom rows), columns 64(w/4)..+63
+      tc_fence_after();
+      {
+        const int row = 32 * (warp & 3) + lane;
+        const int c0 = 64 * (warp >> 2);
+        const uint32_t taddr = tmem + ((uint32_t)(32 * (warp & 3)) << 16) + (uint32_t)c0;
 #pragma unroll
-      for (int nt = 0; nt < 16; ++nt) {
-        const int col = nt * 8 + 2 * t4;
-        const float c0 = bf16_bits_to_f32(p.c[col]), c1 = bf16_bits_to_f32(p.c[col + 1]);
+        for (int q = 0; q < 4; ++q) {
+          float v[16];
+          tmem_ld16(taddr + 16 * q, v);
 #pragma unroll
-        for (int hr = 0; hr < 2; ++hr) {
-          const int row = warp * 16 + g + hr * 8;
-          float v0 = fmaxf(acc[nt][2 * hr] + c0, 0.f), v1 = fmaxf(acc[nt][2 * hr + 1] + c1, 0.f);
-          if (row >= na) v0 = v1 = 0.f;
-          uint16_t h0, l0, h1, l1;
-          split_bf16(v0, h0, l0);
-          split_bf16(v1, h1, l1);
-          const uint32_t off = sw_off(row, col);
-          *reinterpret_cast<uint32_t*>(smem_raw + kOffHhi + off) = h0 | ((uint32_t)h1 << 16);
-          *reinterpret_cast<uint32_t*>(smem_raw + kOffHlo + off) = l0 | ((uint32_t)l1 << 16);
+          for (int hlf = 0; hlf < 2; ++hlf) {
+            float o[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const int col = c0 + 16 * q + 8 * hlf + j;
+              o[j] = row < na ? fmaxf(v[8 * hlf + j] + cvec[col], 0.f) : 0.f;
+            }
+            const uint32_t off = chunk_off(row, (c0 + 16 * q + 8 * hlf) >> 3);
+            split_store8(sm + kOffHhi + off, sm + kOffHlo + off, o);
+          }
         }
       }
+      tc_fence_before();
       __syncthreads();
     }
     // readout: r_m = sum_v h_v (atom order); z_m = ReLU(W1 r_m + c1); y_m = w2 . z_m + c2,
@@ -293,9 +393,9 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const int ab = p.atom_off[mb + mm] - a0, ae = p.atom_off[mb + mm + 1] - a0;
         float t = 0.f;
         for (int v = ab; v < ae; ++v) {
-          const uint32_t off = sw_off(v, f);
-          t += bf16_bits_to_f32(*reinterpret_cast<const uint16_t*>(smem_raw + kOffHhi + off)) +
-               bf16_bits_to_f32(*reinterpret_cast<const uint16_t*>(smem_raw + kOffHlo + off));
+          const uint32_t off = elem_off(v, f);
+          t += bf16_bits_to_f32(*reinterpret_cast<const uint16_t*>(sm + kOffHhi + off)) +
+               bf16_bits_to_f32(*reinterpret_cast<const uint16_t*>(sm + kOffHlo + off));
         }
         rz[mm * 2 * kF + f] = t;
       }
@@ -305,7 +405,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const float* r = rz + mm * 2 * kF;
         float t = bf16_bits_to_f32(p.c1[f]);
         for (int k = 0; k < kF; k += 8) {
-          const uint4 wv = *reinterpret_cast<const uint4*>(smem_raw + kOffW0 + sw_off(f, k));
+          const uint4 wv = *reinterpret_cast<const uint4*>(sm + kOffW0 + chunk_off(f, k >> 3));
           float wf[8];
           unpack8(wv, wf);
 #pragma unroll
@@ -328,7 +428,13 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       __syncthreads();
     }
   }
+  tc_fence_before();
   __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(kTmemCols)
+                 : "memory");
+  }
   if (tid == 0) {
     atomicMax(&p.stamps[1], (unsigned long long)globaltimer());
     if (p.h_stamps) {
