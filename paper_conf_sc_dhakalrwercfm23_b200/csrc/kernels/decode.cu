@@ -16,7 +16,7 @@ int set_attrs_b(int device);
 int decode_smem_bytes(int B, int kmax, int* n_stages) {
   const int fixed = decode_xin_bytes(B, kmax) + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 +
                     8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 128;
-  const int per_stage = kStageBytes + kMaxUnits * B * 4 + kMaxUnits * 4 + 16;
+  const int per_stage = kStageBytes + decode_red_floats(B) * 4 + kMaxUnits * 4 + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;
   if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;

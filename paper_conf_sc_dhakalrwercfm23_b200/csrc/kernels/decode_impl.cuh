@@ -86,6 +86,9 @@ constexpr int kCPG = MX_CPG;                // 256-column chunks per GEMV work u
 // (kacc + partial). Segment widths depend only on the shape, so results stay
 // independent of the partition size.
 constexpr int kTcRows = 8;   // weight rows per tensor-core tile (the n of mma.m16n8k16)
+// kTcGroups tensor-core tiles are in progress at once.
+constexpr int kTcGroups = kConsumerWarps / kTcSplit;
+static_assert(kConsumerWarps % kTcSplit == 0, "tensor-core warp groups must tile the consumers");
 
 struct Phase {
   int kind, layer, R, K, KP, NC, NG, TR;
@@ -212,7 +215,7 @@ __device__ __forceinline__ Smem carve(uint8_t* base, int n_stages, int kmax) {
   p += (size_t)decode_xin_bytes(B, kmax);
   s.zero = p - 64;   // tensor-core path: 64 zero bytes (ldmatrix rows of absent sequences)
   s.red = reinterpret_cast<float*>(p);
-  p += (size_t)n_stages * kMaxUnits * B * 4;
+  p += (size_t)n_stages * decode_red_floats(B) * 4;
   s.cnt = reinterpret_cast<int*>(p);
   p += (size_t)n_stages * kMaxUnits * 4;
   s.att = reinterpret_cast<float*>(p);
@@ -832,7 +835,7 @@ __device__ __forceinline__ void gemv_phase_nr(const DecodeParams& p, const Smem&
     mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
     wait_cyc += MX_CLK() - tw;
     const uint16_t* wt = reinterpret_cast<const uint16_t*>(sm.ring + (size_t)stage * kStageBytes);
-    float* red = sm.red + (size_t)stage * kMaxUnits * B;
+    float* red = sm.red + (size_t)stage * decode_red_floats(B);
     int* cnt = sm.cnt + stage * kMaxUnits;
     for (; u < units; u += kConsumerWarps) {
       const long long tu = MX_CLK();
@@ -1019,16 +1022,22 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
     // Every warp observes every stage fill and arrives on its empty barrier
     // (count kConsumerWarps): a parity wait only tells two consecutive phases
     // apart, so no warp may skip stages and run a full ring ahead. Only the
-    // owner warp computes the tile.
+    // owner group computes the tile.
     const long long tw = MX_CLK();
     mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
     const long long tu = MX_CLK();
     wait_cyc += tu - tw;
-    if (gidx % kConsumerWarps != warp) {
+    // tile gidx belongs to warp group gidx % kTcGroups; its kTcSplit warps split
+    // the K iterations and combine their partials in a fixed order
+    const int grp = gidx % kTcGroups;
+    if (warp / kTcSplit != grp) {
       __syncwarp();
       if (lane == 0) mbar_arrive(&sm.empty[stage]);
     } else {
+      const int q = warp - grp * kTcSplit;
       const int n = min(ph.TR, r1 - r);
+      const int IT = (K + 31) >> 5;
+      const int it0 = (q * IT) / kTcSplit, it1 = ((q + 1) * IT) / kTcSplit;
       const uint32_t wt = smem_u32(sm.ring + (size_t)stage * kStageBytes) + (uint32_t)lr * ws +
                           (uint32_t)lm * 16u;
       float acc[4][4];
@@ -1036,8 +1045,9 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
       for (int c = 0; c < 4; ++c)
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[c][j] = 0.f;
-      uint32_t ah = a_hi, al = a_lo, wp = wt;
-      for (int kk = 0; kk < K; kk += 32) {
+      uint32_t ah = a_hi + (uint32_t)it0 * a_step, al = a_lo + (uint32_t)it0 * a_step;
+      uint32_t wp = wt + (uint32_t)it0 * 64u;
+      for (int kk = it0 * 32; kk < it1 * 32; kk += 32) {
         uint32_t w0, w1, w2, w3, h0, h1, h2, h3, l0, l1, l2, l3;
         ldsm_x4(wp, w0, w1, w2, w3);
         ldsm_x4(ah, h0, h1, h2, h3);
@@ -1061,10 +1071,37 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
       }
       float v0 = (acc[0][0] + acc[1][0]) + (acc[2][0] + acc[3][0]);
       float v1 = (acc[0][1] + acc[1][1]) + (acc[2][1] + acc[3][1]);
+      bool last = true;
+      if (kTcSplit > 1) {
+        // partials -> smem; the warp arriving last sums them in warp order. It
+        // reads them before releasing the stage, so the slot (and its partial
+        // buffer) cannot be reused underneath it.
+        float* red = sm.red + (size_t)stage * decode_red_floats(B);
+        int* cnt = sm.cnt + stage * kMaxUnits;
+        red[(q * 32 + lane) * 2] = v0;
+        red[(q * 32 + lane) * 2 + 1] = v1;
+        __threadfence_block();
+        __syncwarp();
+        int old = 0;
+        if (lane == 0) old = atomicAdd(cnt, 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        last = (old == kTcSplit - 1);
+        if (last) {
+          __threadfence_block();
+          v0 = 0.f;
+          v1 = 0.f;
+#pragma unroll
+          for (int qq = 0; qq < kTcSplit; ++qq) {
+            v0 += red[(qq * 32 + lane) * 2];
+            v1 += red[(qq * 32 + lane) * 2 + 1];
+          }
+          if (lane == 0) *cnt = 0;   // reset for the slot's next round
+        }
+      }
       // all smem reads of the tile are done: release the stage to the producer
       __syncwarp();
       if (lane == 0) mbar_arrive(&sm.empty[stage]);
-      if (gu) {
+      if (last && gu) {
         // tile rows 0..3 = gate rows, 4..7 = up rows: lanes t4 < 2 (gate) fetch
         // the matching up values from lane ^ 2
         const float u0 = __shfl_xor_sync(0xffffffffu, v0, 2);
@@ -1093,7 +1130,7 @@ __device__ __forceinline__ void gemv_phase_tc(const DecodeParams& p, const Smem&
             p.a[b * p.ff + row] = gt / (1.0f + expf(-gt)) * up;
           }
         }
-      } else if (g8 < B) {
+      } else if (last && g8 < B) {
         const int b = g8;
         float vv[2] = {v0, v1};
         unsigned long long kb = 0ull;

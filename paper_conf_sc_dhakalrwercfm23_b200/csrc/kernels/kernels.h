@@ -36,7 +36,21 @@ constexpr int kXinSegBytes = 64 * 1024; // activation staging per K segment (B *
 MX_HD constexpr int decode_seg_cols(int B) { return (kXinSegBytes / (B * 4)) & ~255; }
 // Batch sizes >= kTcMinBatch run the GEMVs on the tensor cores (K7): tiles of
 // 8 weight rows x <= kTcCols columns (one 32 KiB stage with a 16-byte row pad).
-constexpr int kTcMinBatch = 4;
+#ifndef MX_TC_MIN_BATCH
+#define MX_TC_MIN_BATCH 4
+#endif
+constexpr int kTcMinBatch = MX_TC_MIN_BATCH;
+#ifndef MX_TC_SPLIT
+#define MX_TC_SPLIT 4
+#endif
+// A tensor-core tile (one stage) is consumed by kTcSplit warps that split its
+// K iterations.
+constexpr int kTcSplit = MX_TC_SPLIT;
+// floats of per-stage partial-sum space (CUDA-core units: [kMaxUnits][B];
+// tensor-core tiles: the split warps' fragments, [kTcSplit][32 lanes][2])
+MX_HD constexpr int decode_red_floats(int B) {
+  return (B >= kTcMinBatch && kMaxUnits * B < kTcSplit * 64) ? kTcSplit * 64 : kMaxUnits * B;
+}
 constexpr int kTcCols = 2016;
 // Activation staging columns for the widest phase input kmax.
 MX_HD constexpr int decode_xin_cols(int B, int kmax) {
