@@ -223,8 +223,38 @@ def gpu_arm(args, rank, world, local_rank, dist):
     span = s["span_s"]
     wall = h1 - h0
     span, wall = max_over_ranks([span, wall], dist)
+    priv_held = sum(mx.part_query(p)["hbm_used"] for p in parts)
     for p in parts:
         mx.part_destroy(p)
+    # --- N3: the same layout with ONE shared read-only weight copy per GPU ------
+    n3 = None
+    if args.n3:
+        fs = mx.fn_register(mx.decode_desc(cfg, shared_weights=True))
+        sparts = [mx.part_create(gpu, sz, 64 << 20) for sz in LAYOUTS_FILL[n_main]]
+        for p in sparts:
+            mx.fn_load(fs, p)
+        held = sum(mx.part_query(p)["hbm_used"] for p in sparts) + \
+            mx.weight_pool_query(gpu)["used_bytes"]
+        run_batch(mx, fs, sparts, N_TASKS, eq, prompts)   # warm
+        n3_steps = min(args.steps, 2)
+        n3_res = []
+        for _ in range(n3_steps):
+            r, _ = run_batch(mx, fs, sparts, N_TASKS, eq, prompts)
+            n3_res += r
+        s3 = summarize(n3_res, n3_steps)
+        (span3,) = max_over_ranks([s3["span_s"]], dist)
+        v3 = N_TASKS * n3_steps * world / span3
+        n3 = {"tasks_per_s": round(v3, 3), "steps": n3_steps,
+              "hbm_frac_algorithmic": round(bytes_task * v3 / world / 1e9 / peak, 4),
+              "p50_ms": round(s3["p50_ms"], 3), "p99_ms": round(s3["p99_ms"], 3),
+              "hbm_held_gib": round(held / 2**30, 3),
+              "private_hbm_held_gib": round(priv_held / 2**30, 3),
+              "note": "SURVEY.md §8(f) N3: one weight copy per GPU shared by all partitions "
+                      "(MX_FN_SHARED_WEIGHTS); algorithmic bytes still count every "
+                      "partition's weight stream, so L2 hits between partitions can lift "
+                      "the fraction"}
+        for p in sparts:
+            mx.part_destroy(p)
     mx.mx_shutdown()
     if rank != 0:
         return None
@@ -277,6 +307,8 @@ def gpu_arm(args, rank, world, local_rank, dist):
         if base:
             out["ratio_vs_1_partition"] = round(max(d["tasks_per_s"] for d in sweep)
                                                 / base[0]["tasks_per_s"], 3)
+    if n3:
+        out["n3_shared_weights"] = n3
     out["clocks"] = clk.summary()
     if args.cpu_baseline and world == 1:
         out["cpu_baseline"] = cpu_baseline(args)
@@ -345,6 +377,8 @@ def main():
     ap.add_argument("--sweep", default="1,2,4,7,14,18,37",
                     help="comma list of partition counts for the pre-run sweep ('' = none)")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--no-n3", dest="n3", action="store_false",
+                    help="skip the shared-weights (N3) measurement of the chosen layout")
     args = ap.parse_args()
     args.sweep = [int(x) for x in args.sweep.split(",") if x.strip()]
     if args.warmup < 3 and args.impl == "mx":

@@ -136,6 +136,10 @@ static uint64_t ceil_div(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 // Validation
 // ---------------------------------------------------------------------------
 static int validate_fn(const mx_fn_desc& d) {
+  if (d.flags & ~(uint32_t)MX_FN_SHARED_WEIGHTS) {
+    set_error("fn_register: unknown flags 0x%x", d.flags);
+    return MX_EINVAL;
+  }
   if (d.kind == MX_FN_DECODE) {
     const mx_decode_cfg& c = d.dec;
     const int q = c.n_heads * c.head_dim;
@@ -514,6 +518,42 @@ static int alloc_mpnn_slot(Partition& p, FnInst& fi, Slot& s) {
   return MX_OK;
 }
 
+// Seeded bf16 weights (C1) and the RoPE table, generated on device into the
+// instance's weight block (enqueued on `st`, grid of `nct` CTAs).
+static int generate_weights(FnInst& fi, CUstream st, int nct) {
+  const mx_fn_desc& d = fi.fn->desc;
+  uint16_t* w = reinterpret_cast<uint16_t*>(fi.weights);
+  std::vector<int> tids;
+  if (d.kind == MX_FN_DECODE) {
+    const int L = d.dec.n_layers;
+    tids.push_back(0);
+    for (int l = 0; l < L; ++l)
+      for (int k = 0; k <= 8; ++k) tids.push_back(16 * (l + 1) + k);
+    tids.push_back(16 * (L + 1));
+    tids.push_back(16 * (L + 1) + 1);
+  } else {
+    for (int k = 0; k <= 10; ++k)
+      if (!(k >= 1 && k <= 4 && k - 1 >= d.mpnn.n_bond_types)) tids.push_back(k);
+  }
+  for (int tid : tids) {
+    uint64_t off, n;
+    int gain;
+    if (!tensor_span(fi, tid, &off, &n, &gain)) continue;
+    if (mxk::launch_fill_weights(w + off, n, d.weight_seed, (uint32_t)tid, gain, nct, st)) {
+      set_error("weight fill launch failed");
+      return MX_EDEVICE;
+    }
+  }
+  if (d.kind == MX_FN_DECODE) {
+    if (mxk::launch_rope_table(reinterpret_cast<float*>(fi.rope), d.dec.max_seq, d.dec.head_dim,
+                               d.dec.rope_theta, st)) {
+      set_error("rope table launch failed");
+      return MX_EDEVICE;
+    }
+  }
+  return MX_OK;
+}
+
 // Caller holds p.load_mu. Synchronous cold start on the partition's stream.
 static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
   auto it = p.insts.find(fn.id);
@@ -530,50 +570,55 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
     decode_layout(*fi);
   else
     mpnn_layout(*fi);
-  const uint64_t used_before = p.arena.used();
-  int rc = alloc_ptr(p, fi->weight_bytes, &fi->weights);
-  if (rc) return rc;
-  if (d.kind == MX_FN_DECODE) {
-    const mx_decode_cfg& c = d.dec;
-    if ((rc = alloc_ptr(p, (uint64_t)c.max_seq * c.head_dim * 4, &fi->rope))) return rc;
+  int rc = MX_OK;
+  CUstream st = p.cur->stream;
+  const int nct = p.cur->n_ctas;
+  if (d.flags & MX_FN_SHARED_WEIGHTS) {
+    // N3: one copy per GPU in the read-only weight pool, generated by the first
+    // load on this GPU (on the loading partition's SMs) and referenced after.
+    std::lock_guard<std::mutex> wl(gpu.wpool_mu);
+    SharedWeights& sw = gpu.shared_w[fn.id];
+    if (!sw.weights) {
+      if (!gpu.wpool_ready) {
+        if ((rc = gpu.wpool.init(gpu.ordinal, gpu.mem_bytes, gpu.mem_bytes))) {
+          set_error("shared weight pool reservation failed");
+          return rc;
+        }
+        gpu.wpool_ready = true;
+      }
+      CUdeviceptr w = 0, rope = 0;
+      rc = gpu.wpool.alloc(fi->weight_bytes, 256, &w);
+      if (!rc && d.kind == MX_FN_DECODE)
+        rc = gpu.wpool.alloc((uint64_t)d.dec.max_seq * d.dec.head_dim * 4, 256, &rope);
+      if (rc) {
+        set_error("shared weight pool: device memory cannot back %llu more bytes",
+                  (unsigned long long)fi->weight_bytes);
+        return rc;
+      }
+      fi->weights = w;
+      fi->rope = rope;
+      if ((rc = generate_weights(*fi, st, nct))) return rc;
+      CU_TRY(drv().cuStreamSynchronize(st));
+      sw.weights = w;
+      sw.rope = rope;
+      sw.bytes = fi->weight_bytes;
+    }
+    fi->weights = sw.weights;
+    fi->rope = sw.rope;
+    fi->shared_weights = true;
+    ++sw.refs;
+  } else {
+    if ((rc = alloc_ptr(p, fi->weight_bytes, &fi->weights))) return rc;
+    if (d.kind == MX_FN_DECODE) {
+      const mx_decode_cfg& c = d.dec;
+      if ((rc = alloc_ptr(p, (uint64_t)c.max_seq * c.head_dim * 4, &fi->rope))) return rc;
+    }
   }
   for (Slot& s : fi->slots) {
     rc = (d.kind == MX_FN_DECODE) ? alloc_decode_slot(p, *fi, s) : alloc_mpnn_slot(p, *fi, s);
     if (rc) return rc;   // arena bytes stay used (bump allocator); reported by part_query
   }
-  (void)used_before;
-  // generate the weights on the partition's SMs
-  CUstream st = p.cur->stream;
-  const int nct = p.cur->n_ctas;
-  uint16_t* w = reinterpret_cast<uint16_t*>(fi->weights);
-  std::vector<int> tids;
-  if (d.kind == MX_FN_DECODE) {
-    const int L = d.dec.n_layers;
-    tids.push_back(0);
-    for (int l = 0; l < L; ++l)
-      for (int k = 0; k <= 8; ++k) tids.push_back(16 * (l + 1) + k);
-    tids.push_back(16 * (L + 1));
-    tids.push_back(16 * (L + 1) + 1);
-  } else {
-    for (int k = 0; k <= 10; ++k)
-      if (!(k >= 1 && k <= 4 && k - 1 >= d.mpnn.n_bond_types)) tids.push_back(k);
-  }
-  for (int tid : tids) {
-    uint64_t off, n;
-    int gain;
-    if (!tensor_span(*fi, tid, &off, &n, &gain)) continue;
-    if (mxk::launch_fill_weights(w + off, n, d.weight_seed, (uint32_t)tid, gain, nct, st)) {
-      set_error("weight fill launch failed");
-      return MX_EDEVICE;
-    }
-  }
-  if (d.kind == MX_FN_DECODE) {
-    if (mxk::launch_rope_table(reinterpret_cast<float*>(fi->rope), d.dec.max_seq, d.dec.head_dim,
-                               d.dec.rope_theta, st)) {
-      set_error("rope table launch failed");
-      return MX_EDEVICE;
-    }
-  }
+  if (!fi->shared_weights && (rc = generate_weights(*fi, st, nct))) return rc;
   for (Slot& s : fi->slots) {
     if (s.bar) CU_TRY(drv().cuMemsetD8Async(s.bar, 0, 64, st));
     CU_TRY(drv().cuMemsetD8Async(s.stamps, 0, 64, st));
@@ -1103,6 +1148,11 @@ mx_status mx_shutdown(void) {
     }
     g->exec_pool.clear();
   }
+  for (auto& g : L->gpus) {
+    CtxGuard cg(g->primary);
+    if (g->wpool_ready) g->wpool.release();
+    g->shared_w.clear();
+  }
   for (auto& g : L->gpus) drv().cuDevicePrimaryCtxRelease(g->dev);
   g_lib = nullptr;
   delete L;
@@ -1393,6 +1443,20 @@ mx_status fn_load(int32_t fn, int32_t part) {
   std::lock_guard<std::mutex> llk(p->load_mu);
   FnInst* fi = nullptr;
   return load_instance(*g, *p, *f, &fi);
+}
+
+mx_status mx_weight_pool_query(int32_t gpu, uint64_t* used_bytes, int32_t* n_fns) {
+  MX_REQUIRE_INIT();
+  if (!used_bytes || !n_fns) return MX_EINVAL;
+  if (gpu < 0 || gpu >= (int)L->gpus.size()) return MX_ENODEV;
+  Gpu& g = *L->gpus[gpu];
+  std::lock_guard<std::mutex> wl(g.wpool_mu);
+  *used_bytes = g.wpool_ready ? g.wpool.used() : 0;
+  int n = 0;
+  for (auto& kv : g.shared_w)
+    if (kv.second.weights) ++n;
+  *n_fns = n;
+  return MX_OK;
 }
 
 mx_status mx_task_default_cost(const mx_fn_desc* desc, const mx_task_desc* task, uint64_t* out) {

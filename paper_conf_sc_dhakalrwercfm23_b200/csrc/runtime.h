@@ -117,6 +117,14 @@ struct FnInst {
   uint64_t m_off[11] = {};
   Slot slots[2];
   bool loaded = false;
+  bool shared_weights = false;   // weights/rope point into the GPU's weight pool (N3)
+};
+
+// One function's read-only weights in a GPU's shared pool (N3).
+struct SharedWeights {
+  CUdeviceptr weights = 0, rope = 0;
+  uint64_t bytes = 0;
+  int refs = 0;   // partition instances referencing them
 };
 
 struct Partition {
@@ -153,6 +161,12 @@ struct Gpu {
   // part_destroy return execs here and make_exec reuses them.
   std::mutex pool_mu;
   std::multimap<uint64_t, std::unique_ptr<Exec>> exec_pool;
+  // Shared read-only weight pool (MX_FN_SHARED_WEIGHTS, N3): one VMM arena per
+  // GPU, created on first use, quota = device memory; fn id -> its weights.
+  std::mutex wpool_mu;
+  Arena wpool;
+  bool wpool_ready = false;
+  std::map<int, SharedWeights> shared_w;
 };
 
 }  // namespace mx

@@ -20,6 +20,7 @@ MX_OK, MX_ENOENT, MX_EDEVICE, MX_ENOMEM, MX_EBUSY = 0, -2, -5, -12, -16
 MX_ENODEV, MX_EINVAL, MX_ENOSM, MX_ETIMEDOUT, MX_ESTATE = -19, -22, -28, -110, -125
 MX_PART_ANY = -1
 MX_FN_DECODE, MX_FN_MPNN = 1, 2
+MX_FN_SHARED_WEIGHTS = 1
 
 
 class MxError(RuntimeError):
@@ -42,7 +43,7 @@ class MpnnCfgC(C.Structure):
 
 
 class FnDescC(C.Structure):
-    _fields_ = [("kind", C.c_int32), ("reserved", C.c_int32), ("weight_seed", C.c_uint64),
+    _fields_ = [("kind", C.c_int32), ("flags", C.c_uint32), ("weight_seed", C.c_uint64),
                 ("dec", DecodeCfgC), ("mpnn", MpnnCfgC)]
 
 
@@ -90,6 +91,7 @@ _SIGS = {
     "part_query": (C.c_int32, [C.c_int32, C.POINTER(PartInfoC)]),
     "fn_register": (C.c_int32, [C.POINTER(FnDescC), C.POINTER(C.c_int32)]),
     "fn_load": (C.c_int32, [C.c_int32, C.c_int32]),
+    "mx_weight_pool_query": (C.c_int32, [C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_int32)]),
     "fn_submit": (C.c_int32, [C.c_int32, C.POINTER(TaskDescC), C.POINTER(C.c_uint64)]),
     "fn_wait": (C.c_int32, [C.c_uint64, C.c_int64, C.POINTER(ResultC)]),
     "mx_task_default_cost": (C.c_int32, [C.POINTER(FnDescC), C.POINTER(TaskDescC),
@@ -213,18 +215,22 @@ def part_query(part: int) -> dict:
 # Functions and tasks
 # ---------------------------------------------------------------------------
 
-def decode_desc(cfg, max_batch: int = 1, seed: int | None = None) -> FnDescC:
+def decode_desc(cfg, max_batch: int = 1, seed: int | None = None,
+                shared_weights: bool = False) -> FnDescC:
     d = FnDescC()
     d.kind = MX_FN_DECODE
+    d.flags = MX_FN_SHARED_WEIGHTS if shared_weights else 0
     d.weight_seed = cfg.seed if seed is None else seed
     d.dec = DecodeCfgC(cfg.n_layers, cfg.d_model, cfg.n_heads, cfg.n_kv_heads, cfg.head_dim,
                        cfg.d_ff, cfg.vocab, cfg.max_seq, max_batch, cfg.rms_eps, cfg.rope_theta)
     return d
 
 
-def mpnn_desc(cfg, max_mols: int, max_atoms: int, max_edges: int) -> FnDescC:
+def mpnn_desc(cfg, max_mols: int, max_atoms: int, max_edges: int,
+              shared_weights: bool = False) -> FnDescC:
     d = FnDescC()
     d.kind = MX_FN_MPNN
+    d.flags = MX_FN_SHARED_WEIGHTS if shared_weights else 0
     d.weight_seed = cfg.seed
     d.mpnn = MpnnCfgC(cfg.n_atom_types, cfg.n_bond_types, cfg.hidden, cfg.steps, max_mols,
                       max_atoms, max_edges)
@@ -235,6 +241,13 @@ def fn_register(desc: FnDescC) -> int:
     f = C.c_int32()
     _check(lib().fn_register(C.byref(desc), C.byref(f)), "fn_register")
     return f.value
+
+
+def weight_pool_query(gpu: int) -> dict:
+    """Shared read-only weight pool of `gpu` (N3): bytes used and functions held."""
+    used, n = C.c_uint64(0), C.c_int32(0)
+    _check(lib().mx_weight_pool_query(gpu, C.byref(used), C.byref(n)), "mx_weight_pool_query")
+    return {"used_bytes": used.value, "n_fns": n.value}
 
 
 def fn_load(fn: int, part: int):

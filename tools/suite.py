@@ -7,6 +7,7 @@
     python tools/suite.py c4        # D4:  decode + MPNN co-located on 7 partitions vs 1 (WLAW)
     python tools/suite.py c5        # D5:  10k-task farm, 50/50 mix, part_resize every 1000 submissions
     python tools/suite.py modes     # N1:  partitioned vs unpartitioned-concurrent vs time-shared
+    python tools/suite.py n3        # N3:  private vs shared read-only weights (GPT-2s C2, 7B C3)
 
 All inputs are seeded and synthetic (workloads/); weights are generated on the
 device from seeds. Times are device %globaltimer stamps (t_start/t_end of each
@@ -351,6 +352,68 @@ def cmd_modes(a, mx):
             "tasks per point, STATIC placement", "peak_gbs": peak_gbs(), "rows": rows}
 
 
+# ---------------------------------------------------------------------------
+# N3: shared read-only weights across partitions (§7, §6)
+# ---------------------------------------------------------------------------
+
+def cmd_n3(a, mx):
+    """Same closed batches with one weight copy per partition (the paper's
+    one-model-per-process setup) vs ONE copy per GPU referenced by all
+    partitions. Reports tasks/s, algorithmic-bytes HBM fraction (may exceed 1
+    when partitions hit each other's weights in L2), cold-start time of the
+    layout and the HBM held by weights."""
+    rows = []
+    pool_fn = {}   # model -> bytes of its shared copy in the weight pool
+    for cfg, B, layouts, ntask, q_priv, q_sh in (
+            (GPT2S, 1, [int(x) for x in a.gpt2s_layouts.split(",")], a.gpt2s_tasks,
+             512 << 20, 64 << 20),
+            (LLAMA7B, 1, [int(x) for x in a.llama_layouts.split(",")], a.llama_tasks,
+             14 << 30, 1 << 30)):
+        tb = decode_task_bytes(cfg, B, P_LEN, G_LEN)
+        fns = {"private": mx.fn_register(mx.decode_desc(cfg, max_batch=B)),
+               "shared": mx.fn_register(mx.decode_desc(cfg, max_batch=B, shared_weights=True))}
+        for n in layouts:
+            sizes = LAYOUTS_FILL[n]
+            for mode in ("private", "shared"):
+                quota = q_priv if mode == "private" else q_sh
+                if mode == "private" and n * quota > (170 << 30):
+                    rows.append({"model": cfg.name, "partitions": n, "mode": mode,
+                                 "skipped": f"{n} private copies exceed device memory"})
+                    continue
+                fn = fns[mode]
+                pool0 = mx.weight_pool_query(0)["used_bytes"]
+                parts = [mx.part_create(0, s, quota) for s in sizes]
+                t0 = time.perf_counter()
+                for p in parts:
+                    mx.fn_load(fn, p)
+                load_s = time.perf_counter() - t0
+                grown = mx.weight_pool_query(0)["used_bytes"] - pool0
+                if mode == "shared" and grown:
+                    pool_fn[cfg.name] = grown
+                held = sum(mx.part_query(p)["hbm_used"] for p in parts) + \
+                    (pool_fn.get(cfg.name, 0) if mode == "shared" else 0)
+                eq = len(set(sizes)) == 1
+                closed_batch(mx, [(p, mx.decode_task(fn, prompt_tokens(9000 + i, B, P_LEN, cfg.vocab),
+                                                     G_LEN)) for i, p in enumerate(parts)])
+                items = [(parts[(k - 1) % n] if eq else mx.MX_PART_ANY,
+                          mx.decode_task(fn, prompt_tokens(k, B, P_LEN, cfg.vocab), G_LEN))
+                         for k in range(1, ntask + 1)]
+                res, wall = closed_batch(mx, items)
+                sp = span_s(res)
+                rows.append({"model": cfg.name, "partitions": n, "sms": sizes, "mode": mode,
+                             "tasks": ntask, "tasks_per_s": round(ntask / sp, 3),
+                             "gen_tok_per_s": round(ntask * B * G_LEN / sp, 1),
+                             "hbm_frac_algorithmic": round(ntask * tb / sp / 1e9 / peak_gbs(), 4),
+                             "load_s": round(load_s, 3), "hbm_held_gib": round(held / 2**30, 2),
+                             **lat(res)})
+                for p in parts:
+                    mx.part_destroy(p)
+    return {"suite": "N3 shared weights", "workload": "configs[1] GPT-2s and configs[2] 7B "
+            "decode, B=1 P=16 G=32, fill layouts; private = one weight copy per partition, "
+            "shared = one copy per GPU (MX_FN_SHARED_WEIGHTS)", "peak_gbs": peak_gbs(),
+            "rows": rows}
+
+
 def main():
     ap = argparse.ArgumentParser()
     sub = ap.add_subparsers(dest="cmd", required=True)
@@ -371,6 +434,11 @@ def main():
     s.add_argument("--base-tasks", type=int, default=1000)
     s.add_argument("--resize-every", type=int, default=1000)
     s.add_argument("--mol-variants", type=int, default=16)
+    s = sub.add_parser("n3")
+    s.add_argument("--gpt2s-layouts", default="14,18,37")
+    s.add_argument("--gpt2s-tasks", type=int, default=296)
+    s.add_argument("--llama-layouts", default="1,4,7,14")
+    s.add_argument("--llama-tasks", type=int, default=28)
     s = sub.add_parser("modes")
     s.add_argument("--ns", default="1,2,4,7,14")
     s.add_argument("--tasks", type=int, default=140)
