@@ -29,6 +29,14 @@ def prompt_tokens(task_id: int, batch: int, prompt_len: int, vocab: int,
     return out
 
 
+def ip_targets(task_id: int, n_mol: int, seed: int = 0x1B7) -> np.ndarray:
+    """Synthetic training targets ("computed IPs", §3.1 P:109 step (2))
+    for the N4 training step: t_m = ((draw(key(seed, task_id), m) >> 40) / 2^24)
+    * 2 - 1, uniform in [-1, 1), exactly representable in fp32."""
+    r = draw(np.uint64(key(seed, task_id)), np.arange(n_mol, dtype=np.uint64))
+    return ((r >> np.uint64(40)).astype(np.float64) / float(1 << 24) * 2.0 - 1.0).astype(np.float32)
+
+
 # ---------------------------------------------------------------------------
 # Molecules (C1): molecule j of task k uses a sequential counter i over
 # draw(key(seed_g, k*2^20 + j), i):
