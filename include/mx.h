@@ -47,7 +47,17 @@ enum {
   MX_ESTATE = -125     /* library not initialised (or already shut down)              */
 };
 enum { MX_PART_ANY = -1 };           /* fn_submit: let the placement policy choose (C5) */
-enum { MX_FN_DECODE = 1, MX_FN_MPNN = 2 };
+enum { MX_FN_DECODE = 1, MX_FN_MPNN = 2, MX_FN_MPNN_TRAIN = 3 };
+/* MX_FN_MPNN_TRAIN (§3.1 P:109 steps (3)/(7)
+ * "train an ML model that acts as an emulator", §3.4): one SGD step of
+ * the IP emulator per task on the MSE loss over the task's molecules
+ * (reading R10). The instance holds fp32 parameters, initialised from the same
+ * seeded values as MX_FN_MPNN, updated in place; tasks on one partition apply
+ * their steps in seq_in_part order. Uses mx_fn_desc.mpnn; task inputs are the
+ * MPNN CSR arrays plus targets[n_mol] and lr; outputs out_ip[n_mol] = the
+ * predictions BEFORE the update and *out_loss = the loss. fn_read_tensor
+ * returns fp32 values (4 bytes per element) for this kind. Not combinable
+ * with MX_FN_SHARED_WEIGHTS (training state is per instance).             */
 /* mx_fn_desc.flags */
 enum { MX_FN_SHARED_WEIGHTS = 1 };   /* one read-only weight copy per GPU (N3)  */
 enum { MX_INIT_DEFAULT = 0 };
@@ -120,6 +130,11 @@ typedef struct {
   const mx_bond* edges;     /* [n_edges], u, v local to their molecule               */
   float* out_ip;            /* [n_mol]                                              */
   uint64_t cost;            /* placement cost units (C5); 0 = library default       */
+  /* MX_FN_MPNN_TRAIN only                                                     */
+  const float* targets;     /* [n_mol] training targets (the simulated IPs)         */
+  float* out_loss;          /* [1] loss of the step (before the update)             */
+  float lr;                 /* SGD learning rate                                    */
+  int32_t reserved2;
 } mx_task_desc;
 
 typedef struct {

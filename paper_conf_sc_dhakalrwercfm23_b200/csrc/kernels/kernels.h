@@ -153,6 +153,32 @@ int mpnn_smem_bytes();
 int mpnn_pack_tiles(const int* atom_off, const int* edge_off, int n_mol, int* tile_off);
 int launch_mpnn(const MpnnParams& p, void* stream);
 
+// IP-emulator training step (N4): tile forward/backward + SGD apply.
+struct MpnnTrainParams {
+  int T, n_bonds, n_mol, n_params, n_tiles, n_ctas;
+  uint32_t off[11];          // element offsets of the 11 tensors in params (C1 ids)
+  float* params;             // fp32 training state [n_params]
+  float* partials;           // [n_tiles][n_params] per-tile gradients
+  float* hsave;              // [n_tiles][T+1][128][128] saved h^t (feature-major)
+  const int* atom_off;
+  const uint8_t* atom_type;
+  const int* edge_off;
+  const uint32_t* edges;
+  const int* tile_off;
+  const float* targets;      // [n_mol]
+  float* y;                  // [n_mol] device copy of the predictions
+  float* out;                // host-mapped [n_mol + 1]: predictions, loss
+  float lr;
+  unsigned long long* stamps;
+  unsigned long long* h_stamps;
+  unsigned long long done_tag;
+};
+int mpnn_train_smem_bytes();
+uint64_t mpnn_train_tile_scratch_floats(int T);
+int launch_mpnn_train(const MpnnTrainParams& p, void* stream);
+int launch_widen_bf16(float* dst, const uint16_t* src, uint64_t n, int n_ctas, void* stream);
+int mpnn_train_set_attrs(int device);
+
 uint64_t launch_counter();
 
 }  // namespace mxk

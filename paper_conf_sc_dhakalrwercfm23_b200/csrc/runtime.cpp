@@ -140,6 +140,10 @@ static int validate_fn(const mx_fn_desc& d) {
     set_error("fn_register: unknown flags 0x%x", d.flags);
     return MX_EINVAL;
   }
+  if (d.kind == MX_FN_MPNN_TRAIN && (d.flags & MX_FN_SHARED_WEIGHTS)) {
+    set_error("fn_register: a training function's parameters are per-instance state");
+    return MX_EINVAL;
+  }
   if (d.kind == MX_FN_DECODE) {
     const mx_decode_cfg& c = d.dec;
     const int q = c.n_heads * c.head_dim;
@@ -176,7 +180,7 @@ static int validate_fn(const mx_fn_desc& d) {
     }
     return MX_OK;
   }
-  if (d.kind == MX_FN_MPNN) {
+  if (d.kind == MX_FN_MPNN || d.kind == MX_FN_MPNN_TRAIN) {
     const mx_mpnn_cfg& m = d.mpnn;
     if (m.hidden != 128 || m.steps < 1 || m.n_bond_types < 1 || m.n_bond_types > 4 ||
         m.n_atom_types < 1 || m.n_atom_types > 256 || m.max_mols < 1 || m.max_atoms < 1 ||
@@ -209,6 +213,10 @@ static int validate_task(const mx_fn_desc& d, const mx_task_desc& t) {
   if (t.n_mol < 1 || t.n_mol > m.max_mols || !t.atom_off || !t.atom_type || !t.edge_off ||
       (t.n_edges > 0 && !t.edges) || !t.out_ip) {
     set_error("mpnn task: bad sizes or null buffers");
+    return MX_EINVAL;
+  }
+  if (d.kind == MX_FN_MPNN_TRAIN && (!t.targets || !t.out_loss || !(t.lr == t.lr))) {
+    set_error("mpnn training task: needs targets, out_loss and a finite lr");
     return MX_EINVAL;
   }
   if (t.atom_off[0] != 0 || t.edge_off[0] != 0 || t.atom_off[t.n_mol] != t.n_atoms ||
@@ -249,7 +257,8 @@ static uint64_t default_cost(const mx_fn_desc& d, const mx_task_desc& t) {
     fl += mpnn_mol_flops(n, eb + (size_t)t.edge_off[i] * 6, ne, (uint64_t)d.mpnn.hidden,
                          (uint64_t)d.mpnn.steps);
   }
-  return ceil_div(fl, 75000);
+  // training: forward + backward ~ 3x the forward contractions (N4)
+  return ceil_div(d.kind == MX_FN_MPNN_TRAIN ? 3 * fl : fl, 75000);
 }
 
 // ---------------------------------------------------------------------------
@@ -421,7 +430,7 @@ static void mpnn_layout(FnInst& fi) {
 static bool tensor_span(const FnInst& fi, int tid, uint64_t* off, uint64_t* n, int* is_gain) {
   const mx_fn_desc& d = fi.fn->desc;
   *is_gain = 0;
-  if (d.kind == MX_FN_MPNN) {
+  if (d.kind == MX_FN_MPNN || d.kind == MX_FN_MPNN_TRAIN) {
     const uint64_t F = d.mpnn.hidden;
     const uint64_t sizes[11] = {(uint64_t)d.mpnn.n_atom_types * F, F * F, F * F, F * F, F * F,
                                 F * F, F, F * F, F, F, 1};
@@ -512,6 +521,17 @@ static int alloc_mpnn_slot(Partition& p, FnInst& fi, Slot& s) {
   s.err = s.stamps + 16;
   s.h_in_bytes = align_up((M + 1) * 4, 64) * 3 + align_up(NA, 64) + align_up(NE * 6, 64) + 64;
   s.h_out_bytes = M * 4;
+  if (fi.fn->desc.kind == MX_FN_MPNN_TRAIN) {
+    // tiles hold >= 4 molecules (<= 32 atoms each) except the last
+    const uint64_t tiles = (M + 3) / 4 + 1;
+    if ((rc = alloc_ptr(p, M * 4, &s.targets))) return rc;
+    if ((rc = alloc_ptr(p, M * 4, &s.y))) return rc;
+    if ((rc = alloc_ptr(p, tiles * fi.n_params * 4, &s.partials))) return rc;
+    if ((rc = alloc_ptr(p, tiles * mxk::mpnn_train_tile_scratch_floats(m.steps) * 4, &s.hsave)))
+      return rc;
+    s.h_in_bytes += align_up(M * 4, 64);
+    s.h_out_bytes = (M + 1) * 4;
+  }
   if ((rc = host_alloc(s.h_in_bytes, &s.h_in, &s.d_in))) return rc;
   if ((rc = host_alloc(s.h_out_bytes, &s.h_out, &s.d_out))) return rc;
   if ((rc = host_alloc(64, reinterpret_cast<void**>(&s.h_stamps), &s.d_stamps))) return rc;
@@ -609,6 +629,10 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
     ++sw.refs;
   } else {
     if ((rc = alloc_ptr(p, fi->weight_bytes, &fi->weights))) return rc;
+    if (d.kind == MX_FN_MPNN_TRAIN) {
+      fi->n_params = fi->weight_bytes / 2;
+      if ((rc = alloc_ptr(p, fi->n_params * 4, &fi->params))) return rc;
+    }
     if (d.kind == MX_FN_DECODE) {
       const mx_decode_cfg& c = d.dec;
       if ((rc = alloc_ptr(p, (uint64_t)c.max_seq * c.head_dim * 4, &fi->rope))) return rc;
@@ -619,6 +643,15 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
     if (rc) return rc;   // arena bytes stay used (bump allocator); reported by part_query
   }
   if (!fi->shared_weights && (rc = generate_weights(*fi, st, nct))) return rc;
+  if (d.kind == MX_FN_MPNN_TRAIN) {
+    // fp32 training state, widened exactly from the seeded bf16 values (N4)
+    if (mxk::launch_widen_bf16(reinterpret_cast<float*>(fi->params),
+                               reinterpret_cast<const uint16_t*>(fi->weights), fi->n_params, nct,
+                               st)) {
+      set_error("parameter widening launch failed");
+      return MX_EDEVICE;
+    }
+  }
   for (Slot& s : fi->slots) {
     if (s.bar) CU_TRY(drv().cuMemsetD8Async(s.bar, 0, 64, st));
     CU_TRY(drv().cuMemsetD8Async(s.stamps, 0, 64, st));
@@ -774,7 +807,39 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.n_ctas = e->n_ctas;
     k.tile_off = reinterpret_cast<const int*>(s.tile_off);
     k.n_tiles = n_tiles;
-    if (mxk::launch_mpnn(k, st)) {
+    if (t->kind == MX_FN_MPNN_TRAIN) {
+      float* ht = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(h5) +
+                                           align_up((size_t)(t->n_mol + 1) * 4, 64));
+      memcpy(ht, t->targets.data(), (size_t)t->n_mol * 4);
+      CU_TRY(drv().cuMemcpyHtoDAsync(s.targets, ht, (size_t)t->n_mol * 4, st));
+      mxk::MpnnTrainParams q{};
+      q.T = m.steps;
+      q.n_bonds = m.n_bond_types;
+      q.n_mol = t->n_mol;
+      q.n_params = (int)fi->n_params;
+      q.n_tiles = n_tiles;
+      q.n_ctas = e->n_ctas;
+      for (int i = 0; i < 11; ++i) q.off[i] = (uint32_t)fi->m_off[i];
+      q.params = reinterpret_cast<float*>(fi->params);
+      q.partials = reinterpret_cast<float*>(s.partials);
+      q.hsave = reinterpret_cast<float*>(s.hsave);
+      q.atom_off = k.atom_off;
+      q.atom_type = k.atom_type;
+      q.edge_off = k.edge_off;
+      q.edges = k.edges;
+      q.tile_off = k.tile_off;
+      q.targets = reinterpret_cast<const float*>(s.targets);
+      q.y = reinterpret_cast<float*>(s.y);
+      q.out = reinterpret_cast<float*>(s.d_out);
+      q.lr = t->lr;
+      q.stamps = k.stamps;
+      q.h_stamps = k.h_stamps;
+      q.done_tag = t->id;
+      if (mxk::launch_mpnn_train(q, st)) {
+        set_error("mpnn training launch failed");
+        return MX_EDEVICE;
+      }
+    } else if (mxk::launch_mpnn(k, st)) {
       set_error("mpnn launch failed");
       return MX_EDEVICE;
     }
@@ -816,6 +881,8 @@ static void finish_task(Gpu& gpu, Task* t, bool dev_ok) {
     }
   } else {
     memcpy(t->out_ip, s.h_out, (size_t)t->n_mol * 4);
+    if (t->kind == MX_FN_MPNN_TRAIN)
+      memcpy(t->out_loss, static_cast<uint8_t*>(s.h_out) + (size_t)t->n_mol * 4, 4);
   }
   t->t_start = (uint64_t)((int64_t)st[0] + gpu.clock_offset);
   t->t_end = (uint64_t)((int64_t)st[1] + gpu.clock_offset);
@@ -1009,7 +1076,8 @@ static int init_gpu(Gpu& gpu) {
       return MX_EDEVICE;
     }
   gpu.remainder = gpu.sm_total - gpu.n_groups * gpu.group_size;
-  if (mxk::decode_set_attrs(gpu.dev) || mxk::mpnn_set_attrs(gpu.dev)) {
+  if (mxk::decode_set_attrs(gpu.dev) || mxk::mpnn_set_attrs(gpu.dev) ||
+      mxk::mpnn_train_set_attrs(gpu.dev)) {
     set_error("setting kernel shared-memory attributes failed");
     return MX_EDEVICE;
   }
@@ -1504,6 +1572,11 @@ mx_status fn_submit(int32_t part, const mx_task_desc* task, uint64_t* out_task) 
     const uint8_t* eb = reinterpret_cast<const uint8_t*>(task->edges);
     t->edges.assign(eb, eb + (size_t)t->n_edges * 6);
     t->out_ip = task->out_ip;
+    if (t->kind == MX_FN_MPNN_TRAIN) {
+      t->targets.assign(task->targets, task->targets + t->n_mol);
+      t->lr = task->lr;
+      t->out_loss = task->out_loss;
+    }
   }
   Task* raw = t.get();
   Partition* p = nullptr;
@@ -1633,12 +1706,16 @@ mx_status fn_read_tensor(int32_t fn, int32_t part, int32_t tensor_id, void* host
   }
   uint64_t off, n;
   int gain;
-  if (!tensor_span(*it->second, tensor_id, &off, &n, &gain) || bytes > n * 2) {
+  const bool f32 = it->second->fn->desc.kind == MX_FN_MPNN_TRAIN;   // fp32 training state
+  if (!tensor_span(*it->second, tensor_id, &off, &n, &gain) || bytes > n * (f32 ? 4 : 2)) {
     set_error("bad tensor id %d or size", tensor_id);
     return MX_EINVAL;
   }
   CtxGuard cg(g->primary);
-  CU_TRY(drv().cuMemcpyDtoH(host, it->second->weights + off * 2, bytes));
+  if (f32)
+    CU_TRY(drv().cuMemcpyDtoH(host, it->second->params + off * 4, bytes));
+  else
+    CU_TRY(drv().cuMemcpyDtoH(host, it->second->weights + off * 2, bytes));
   return MX_OK;
 }
 

@@ -61,6 +61,10 @@ struct Task {
   std::vector<int32_t> atom_off, edge_off;
   std::vector<uint8_t> atom_type, edges;
   float* out_ip = nullptr;
+  // mpnn training step (N4)
+  std::vector<float> targets;
+  float lr = 0.f;
+  float* out_loss = nullptr;
   // execution
   bool ready = false;
   FnInst* inst = nullptr;
@@ -84,6 +88,8 @@ struct Slot {
               logits = 0;
   // mpnn
   CUdeviceptr atom_off = 0, atom_type = 0, edge_off = 0, edges = 0, out = 0, tile_off = 0;
+  // mpnn training (N4)
+  CUdeviceptr targets = 0, y = 0, partials = 0, hsave = 0;
   // common
   CUdeviceptr bar = 0, stamps = 0, err = 0;
   uint64_t bar_count = 0;
@@ -118,6 +124,8 @@ struct FnInst {
   Slot slots[2];
   bool loaded = false;
   bool shared_weights = false;   // weights/rope point into the GPU's weight pool (N3)
+  CUdeviceptr params = 0;        // MX_FN_MPNN_TRAIN: fp32 training state (N4)
+  uint64_t n_params = 0;
 };
 
 // One function's read-only weights in a GPU's shared pool (N3).

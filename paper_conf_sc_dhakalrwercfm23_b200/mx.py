@@ -19,7 +19,7 @@ LIB_PATH = os.environ.get("MX_LIB") or os.path.join(_HERE, "libmx.so")
 MX_OK, MX_ENOENT, MX_EDEVICE, MX_ENOMEM, MX_EBUSY = 0, -2, -5, -12, -16
 MX_ENODEV, MX_EINVAL, MX_ENOSM, MX_ETIMEDOUT, MX_ESTATE = -19, -22, -28, -110, -125
 MX_PART_ANY = -1
-MX_FN_DECODE, MX_FN_MPNN = 1, 2
+MX_FN_DECODE, MX_FN_MPNN, MX_FN_MPNN_TRAIN = 1, 2, 3
 MX_FN_SHARED_WEIGHTS = 1
 
 
@@ -53,7 +53,8 @@ class TaskDescC(C.Structure):
                 ("out_logits", C.c_void_p), ("n_mol", C.c_int32), ("n_atoms", C.c_int32),
                 ("n_edges", C.c_int32), ("reserved", C.c_int32), ("atom_off", C.c_void_p),
                 ("atom_type", C.c_void_p), ("edge_off", C.c_void_p), ("edges", C.c_void_p),
-                ("out_ip", C.c_void_p), ("cost", C.c_uint64)]
+                ("out_ip", C.c_void_p), ("cost", C.c_uint64), ("targets", C.c_void_p),
+                ("out_loss", C.c_void_p), ("lr", C.c_float), ("reserved2", C.c_int32)]
 
 
 class ResultC(C.Structure):
@@ -263,7 +264,7 @@ class Task:
         self.desc.fn = fn
         self.keep = []
         self.id = 0
-        self.tokens = self.logits = self.ip = None
+        self.tokens = self.logits = self.ip = self.loss = None
 
 
 def decode_task(fn: int, prompt: np.ndarray, gen_len: int, want_logits: bool = False,
@@ -300,6 +301,32 @@ def mpnn_task(fn: int, mol: dict, cost: int = 0) -> Task:
     d.cost = cost
     t.keep = [ao, at, eo, ed]
     return t
+
+
+def mpnn_train_desc(cfg, max_mols: int, max_atoms: int, max_edges: int) -> FnDescC:
+    """IP-emulator training step function (N4): fp32 parameters per instance."""
+    d = mpnn_desc(cfg, max_mols, max_atoms, max_edges)
+    d.kind = MX_FN_MPNN_TRAIN
+    return d
+
+
+def mpnn_train_task(fn: int, mol: dict, targets: np.ndarray, lr: float, cost: int = 0) -> Task:
+    """One SGD step on the molecules `mol` with `targets`; after fn_wait,
+    task.ip = predictions before the update, task.loss[0] = the loss."""
+    t = mpnn_task(fn, mol, cost)
+    tg = np.ascontiguousarray(targets, dtype=np.float32)
+    assert tg.shape == t.ip.shape
+    t.loss = np.zeros(1, dtype=np.float32)
+    t.desc.targets, t.desc.out_loss, t.desc.lr = _ptr(tg), _ptr(t.loss), float(lr)
+    t.keep.append(tg)
+    return t
+
+
+def fn_read_params(fn: int, part: int, tensor_id: int, n_elems: int) -> np.ndarray:
+    """fp32 training state of a MX_FN_MPNN_TRAIN instance (tensor ids as C1)."""
+    out = np.empty(n_elems, dtype=np.float32)
+    _check(lib().fn_read_tensor(fn, part, tensor_id, _ptr(out), n_elems * 4), "fn_read_tensor")
+    return out
 
 
 def fn_submit(part: int, task: Task) -> int:

@@ -1,0 +1,110 @@
+"""GPU parity of the IP-emulator training step (PAPER.md
+§3.1 P:109 steps (3)/(7), §3.4) against oracle/mpnn_train.py on the
+same seeded parameters, molecules and targets (reading R10: MSE loss, one SGD
+step). Tolerances as C7: predictions within 2e-2 of max |y|, the loss within
+2e-2 relative, and every tensor's UPDATE (theta_new - theta_old) within 2e-2 of
+the largest oracle update of that tensor."""
+import numpy as np
+import pytest
+
+from oracle import mpnn_train as ot
+from workloads.configs import MPNN
+from workloads.inputs import molecules, ip_targets
+from workloads.weights import mpnn_weights
+
+pytestmark = pytest.mark.gpu
+
+TOL = 2e-2
+TIDS = {"e_atom": 0, "w_b": 1, "u": 5, "c": 6, "w1": 7, "c1": 8, "w2": 9, "c2": 10}
+
+
+def _read(mxlib, fn, part, w_like):
+    out = {}
+    for k, tid in TIDS.items():
+        if k == "w_b":
+            arrs = [mxlib.fn_read_params(fn, part, 1 + b, 128 * 128).reshape(128, 128)
+                    for b in range(MPNN.n_bond_types)]
+            out[k] = np.stack(arrs).astype(np.float64)
+        else:
+            n = int(np.asarray(w_like[k]).size)
+            out[k] = mxlib.fn_read_params(fn, part, tid, n).reshape(np.asarray(w_like[k]).shape)
+            out[k] = out[k].astype(np.float64)
+    return out
+
+
+def _check_update(old, gpu_new, orc_new):
+    for k in ot.PARAMS:
+        d_g = np.asarray(gpu_new[k]) - np.asarray(old[k], dtype=np.float64)
+        d_o = np.asarray(orc_new[k]) - np.asarray(old[k], dtype=np.float64)
+        scale = float(np.max(np.abs(d_o)))
+        if scale == 0.0:
+            assert float(np.max(np.abs(d_g))) == 0.0, k
+            continue
+        err = float(np.max(np.abs(d_g - d_o))) / scale
+        assert err <= TOL, (k, err)
+
+
+def test_train_step_parity_multi_tile(mxlib, parts):
+    p = parts(20, hbm=512 << 20)
+    M = 96
+    fn = mxlib.fn_register(mxlib.mpnn_train_desc(MPNN, M, M * 32, M * 64))
+    mxlib.fn_load(fn, p)
+    w0 = mpnn_weights(MPNN)
+    start = _read(mxlib, fn, p, w0)
+    for k in ot.PARAMS:   # fp32 state = the seeded bf16-exact values
+        assert np.array_equal(start[k], np.asarray(w0[k], dtype=np.float64)), k
+    mol, tg, lr = molecules(21, M), ip_targets(21, M), 0.5
+    t = mxlib.mpnn_train_task(fn, mol, tg, lr)
+    mxlib.fn_submit(p, t)
+    assert mxlib.fn_wait(t)["status"] == 0
+    new_o, loss_o, ys_o, _ = ot.train_step(w0, mol, tg, MPNN.steps, lr)
+    assert np.max(np.abs(t.ip - ys_o)) / np.max(np.abs(ys_o)) <= TOL
+    assert abs(float(t.loss[0]) - loss_o) / loss_o <= TOL
+    _check_update(w0, _read(mxlib, fn, p, w0), new_o)
+
+
+def test_three_steps_fifo_and_partition_size_independence(mxlib, parts):
+    """Three tasks on one partition = three sequential SGD steps (seq_in_part
+    order); the same steps on a 4x larger partition give bit-identical
+    parameters (tile-order gradient reduction)."""
+    M = 40
+    pa, pb = parts(8, hbm=256 << 20), parts(32, hbm=256 << 20)
+    fa = mxlib.fn_register(mxlib.mpnn_train_desc(MPNN, M, M * 32, M * 64))
+    w = {k: np.asarray(v, dtype=np.float64) for k, v in mpnn_weights(MPNN).items()}
+    w0 = dict(w)
+    losses_gpu = {pa: [], pb: []}
+    for part in (pa, pb):
+        ts = []
+        for s in range(3):
+            t = mxlib.mpnn_train_task(fa, molecules(30 + s, M), ip_targets(30 + s, M), 0.5)
+            mxlib.fn_submit(part, t)
+            ts.append(t)
+        for t in ts:
+            assert mxlib.fn_wait(t)["status"] == 0
+            losses_gpu[part].append(float(t.loss[0]))
+    losses_o = []
+    for s in range(3):
+        w, loss, _, _ = ot.train_step(w, molecules(30 + s, M), ip_targets(30 + s, M), MPNN.steps, 0.5)
+        losses_o.append(loss)
+    for lg, lo in zip(losses_gpu[pa], losses_o):
+        assert abs(lg - lo) / lo <= TOL, (lg, lo)
+    assert losses_gpu[pa] == losses_gpu[pb]
+    ra, rb = _read(mxlib, fa, pa, w0), _read(mxlib, fa, pb, w0)
+    for k in ot.PARAMS:
+        assert np.array_equal(ra[k], rb[k]), k
+    _check_update(w0, ra, w)
+
+
+def test_train_rejects_shared_weights_and_missing_targets(mxlib, parts):
+    d = mxlib.mpnn_train_desc(MPNN, 8, 8 * 32, 8 * 64)
+    d.flags = mxlib.MX_FN_SHARED_WEIGHTS
+    with pytest.raises(mxlib.MxError) as e:
+        mxlib.fn_register(d)
+    assert e.value.code == mxlib.MX_EINVAL
+    p = parts(8, hbm=128 << 20)
+    fn = mxlib.fn_register(mxlib.mpnn_train_desc(MPNN, 8, 8 * 32, 8 * 64))
+    t = mxlib.mpnn_train_task(fn, molecules(1, 8), ip_targets(1, 8), 0.1)
+    t.desc.targets = None
+    with pytest.raises(mxlib.MxError) as e:
+        mxlib.fn_submit(p, t)
+    assert e.value.code == mxlib.MX_EINVAL
