@@ -27,13 +27,21 @@
 #include "common.cuh"
 #include "kernels.h"
 #include "launch.cuh"
+#ifdef MX_MPNN_PROF
+#include <cstdio>
+#endif
 
 namespace mxk {
 
 constexpr int kF = 128;
 constexpr int kTileAtoms = 128;
 constexpr int kTileEdges = 512;
-constexpr int kMpnnThreads = 256;
+#ifndef MX_MPNN_THREADS
+#define MX_MPNN_THREADS 512
+#endif
+constexpr int kMpnnThreads = MX_MPNN_THREADS;   // 16 warps: the gathers are smem-latency bound
+constexpr int kEpiCols = kF / (kMpnnThreads / 128);   // accumulator columns per epilogue warp
+static_assert(kMpnnThreads % 128 == 0 && kEpiCols % 16 == 0, "epilogue warp mapping");
 constexpr int kMatBytes = kF * kF * 2;        // one 128x128 bf16 operand (two 16 KiB halves)
 constexpr int kHalfBytes = kMatBytes / 2;     // [128 rows][64 cols] SWIZZLE_128B region
 constexpr int kTmemCols = 128;                // fp32 accumulator 128 lanes x 128 columns
@@ -55,7 +63,11 @@ constexpr int kOffC = kOffR + kReadoutMols * 2 * kF * 4;       // float [kF]: bi
 constexpr int kOffRed = kOffC + kF * 4;                        // float [16]
 constexpr int kOffBar = kOffRed + 64;                          // uint64 mbarrier (MMA done)
 constexpr int kOffTmem = kOffBar + 8;                          // uint32 TMEM base address
-constexpr int kMpnnSmem = kOffTmem + 8 + 1024;                 // + alignment slack
+constexpr int kOffOff4 = kOffTmem + 8;                         // int [kTileAtoms][5]: per-type ranges
+constexpr int kOffMoff = kOffOff4 + kTileAtoms * 5 * 4;        // int [kTileAtoms+4]: tile-local atom offsets
+constexpr int kOffEoff = kOffMoff + (kTileAtoms + 4) * 4;      // int [kTileAtoms+4]: tile-local edge offsets
+constexpr int kOffType = kOffEoff + (kTileAtoms + 4) * 4;      // uint8 [kTileAtoms]: atom types
+constexpr int kMpnnSmem = kOffType + kTileAtoms + 1024;        // + alignment slack
 
 int mpnn_smem_bytes() { return kMpnnSmem; }
 
@@ -159,30 +171,34 @@ __device__ __forceinline__ void split_store8(uint8_t* hi_dst, uint8_t* lo_dst, c
   *reinterpret_cast<uint4*>(lo_dst) = pl;
 }
 
-// s_b[v] = sum over type-b bonds of v of h[neighbour] (neighbour-list order),
-// written as a hi/lo operand; padded rows are 0.
-__device__ __forceinline__ void build_s(uint8_t* sm, const int* nbr_off, const int* nbr, int na,
+// s_b[v] = sum over type-b bonds of v of the neighbour's h (edge order), written
+// as a hi/lo operand; padded rows and atoms without a type-b bond are 0. The
+// neighbour list is bucketed by bond type (off4[v][b] .. off4[v][b+1]), so an
+// (atom, type) pair without bonds costs two zero stores.
+__device__ __forceinline__ void build_s(uint8_t* sm, const int* off4, const int* nbr, int na,
                                         int b, int tid) {
   for (int i = tid; i < kTileAtoms * 16; i += kMpnnThreads) {
     const int v = i >> 4, ch = i & 15;
+    const uint32_t off = chunk_off(v, ch);
+    const int q0 = (v < na) ? off4[v * 5 + b] : 0, q1 = (v < na) ? off4[v * 5 + b + 1] : 0;
+    if (q0 == q1) {
+      *reinterpret_cast<uint4*>(sm + kOffShi + off) = make_uint4(0, 0, 0, 0);
+      *reinterpret_cast<uint4*>(sm + kOffSlo + off) = make_uint4(0, 0, 0, 0);
+      continue;
+    }
     float sacc[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) sacc[j] = 0.f;
-    if (v < na) {
-      for (int q = nbr_off[v]; q < nbr_off[v + 1]; ++q) {
-        const int nb = nbr[q];
-        if ((nb & 3) != b) continue;
-        const uint32_t off = chunk_off(nb >> 2, ch);
-        const uint4 hh = *reinterpret_cast<const uint4*>(sm + kOffHhi + off);
-        const uint4 hl = *reinterpret_cast<const uint4*>(sm + kOffHlo + off);
-        float fh[8], fl[8];
-        unpack8(hh, fh);
-        unpack8(hl, fl);
+    for (int q = q0; q < q1; ++q) {
+      const uint32_t hoff = chunk_off(nbr[q] >> 2, ch);
+      const uint4 hh = *reinterpret_cast<const uint4*>(sm + kOffHhi + hoff);
+      const uint4 hl = *reinterpret_cast<const uint4*>(sm + kOffHlo + hoff);
+      float fh[8], fl[8];
+      unpack8(hh, fh);
+      unpack8(hl, fl);
 #pragma unroll
-        for (int j = 0; j < 8; ++j) sacc[j] += fh[j] + fl[j];
-      }
+      for (int j = 0; j < 8; ++j) sacc[j] += fh[j] + fl[j];
     }
-    const uint32_t off = chunk_off(v, ch);
     split_store8(sm + kOffShi + off, sm + kOffSlo + off, sacc);
   }
 }
@@ -199,6 +215,10 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   int2* mol_e = reinterpret_cast<int2*>(sm + kOffMolE);
   int* nbr_off = reinterpret_cast<int*>(sm + kOffNbrOff);
   int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
+  int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
+  int* moff = reinterpret_cast<int*>(sm + kOffMoff);
+  int* eoff = reinterpret_cast<int*>(sm + kOffEoff);
+  uint8_t* typ = sm + kOffType;
   float* rz = reinterpret_cast<float*>(sm + kOffR);
   float* cvec = reinterpret_cast<float*>(sm + kOffC);
   float* red = reinterpret_cast<float*>(sm + kOffRed);
@@ -228,41 +248,48 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   uint32_t mma_phase = 0;
   const uint32_t bar_s = smem_u32(mma_bar);
 
+#ifdef MX_MPNN_PROF
+  long long c_setup = 0, c_steps = 0, c_read = 0, c_build = 0, c_mma = 0;
+#endif
   for (int tile = blockIdx.x; tile < p.n_tiles; tile += p.n_ctas) {
+#ifdef MX_MPNN_PROF
+    long long tp0 = clock64();
+#endif
     const int m0 = p.tile_off[tile], m1 = p.tile_off[tile + 1];
     const int a0 = p.atom_off[m0], na = p.atom_off[m1] - a0;
     const int e0 = p.edge_off[m0], ne = p.edge_off[m1] - e0;
-    // atom -> its molecule's edge range (tile-local); edges in tile-local atom ids
-    for (int i = tid; i < kTileAtoms; i += kMpnnThreads) mol_e[i] = make_int2(0, 0);
-    __syncthreads();
-    for (int m = m0 + tid; m < m1; m += kMpnnThreads) {
-      const int ab = p.atom_off[m] - a0, ae = p.atom_off[m + 1] - a0;
-      const int eb0 = p.edge_off[m] - e0, ee = p.edge_off[m + 1] - e0;
-      for (int v = ab; v < ae; ++v) mol_e[v] = make_int2(eb0, ee);
+    // tile-local molecule offsets, atom types and raw edges: independent loads,
+    // one round trip
+    const int nmt = m1 - m0;
+    for (int j = tid; j <= nmt; j += kMpnnThreads) {
+      moff[j] = p.atom_off[m0 + j] - a0;
+      eoff[j] = p.edge_off[m0 + j] - e0;
     }
+    for (int i = tid; i < na; i += kMpnnThreads) typ[i] = p.atom_type[a0 + i];
     for (int i = tid; i < ne; i += kMpnnThreads) {
       const uint8_t* e = eb + (size_t)(e0 + i) * 6;
-      // local atom ids -> tile ids: add the molecule's first atom (found below)
       ed[i] = make_int4((int)(int16_t)(e[0] | (e[1] << 8)), (int)(int16_t)(e[2] | (e[3] << 8)),
                         (int)e[4], 0);
     }
     __syncthreads();
+    // atom -> its molecule's edge range; edges -> tile-local atom ids (binary
+    // search over the staged edge offsets)
+    for (int j = tid; j < nmt; j += kMpnnThreads)
+      for (int v = moff[j]; v < moff[j + 1]; ++v) mol_e[v] = make_int2(eoff[j], eoff[j + 1]);
     for (int i = tid; i < ne; i += kMpnnThreads) {
-      // molecule of edge i: binary search over the tile's edge offsets
-      int lo = m0, hi = m1 - 1;
+      int lo = 0, hi = nmt - 1;
       while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
-        if (p.edge_off[mid] - e0 <= i) lo = mid; else hi = mid - 1;
+        if (eoff[mid] <= i) lo = mid; else hi = mid - 1;
       }
-      const int base = p.atom_off[lo] - a0;
-      ed[i].x += base;
-      ed[i].y += base;
+      ed[i].x += moff[lo];
+      ed[i].y += moff[lo];
     }
     // h0 = E_atom[type] (bf16-exact: hi = value, lo = 0); padded rows = 0
     for (int i = tid; i < kTileAtoms * kF / 8; i += kMpnnThreads) {
       const int row = i >> 4, ch = i & 15;
       uint4 hv = make_uint4(0, 0, 0, 0);
-      if (row < na) hv = *reinterpret_cast<const uint4*>(p.e_atom + (size_t)p.atom_type[a0 + row] * kF + ch * 8);
+      if (row < na) hv = *reinterpret_cast<const uint4*>(p.e_atom + (size_t)typ[row] * kF + ch * 8);
       const uint32_t off = chunk_off(row, ch);
       *reinterpret_cast<uint4*>(sm + kOffHhi + off) = hv;
       *reinterpret_cast<uint4*>(sm + kOffHlo + off) = make_uint4(0, 0, 0, 0);
@@ -288,23 +315,48 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       int base = 0;
       for (int w = 0; w < warp && w < 4; ++w) base += __float_as_int(red[w]);
       if (v < kTileAtoms) {
-        int pos = base + incl - deg;
+        const int pos = base + incl - deg;
         nbr_off[v] = pos;
         if (v == kTileAtoms - 1) nbr_off[kTileAtoms] = base + incl;
         if (v < na) {
+          // bucket v's neighbours by bond type, edge order inside a bucket
           const int2 er = mol_e[v];
+          int cnt = 0;   // 8-bit count per bond type
           for (int e = er.x; e < er.y; ++e) {
             const int4 E = ed[e];
-            if (E.x == v) nbr[pos++] = (E.y << 2) | E.z;
-            if (E.y == v) nbr[pos++] = (E.x << 2) | E.z;
+            cnt += ((E.x == v) + (E.y == v)) << (8 * E.z);
+          }
+          int o0 = pos, o1 = o0 + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255),
+              o3 = o2 + ((cnt >> 16) & 255);
+          off4[v * 5 + 0] = o0;
+          off4[v * 5 + 1] = o1;
+          off4[v * 5 + 2] = o2;
+          off4[v * 5 + 3] = o3;
+          off4[v * 5 + 4] = pos + deg;
+          for (int e = er.x; e < er.y; ++e) {
+            const int4 E = ed[e];
+            for (int side = 0; side < 2; ++side) {
+              const int me = side ? E.y : E.x, other = side ? E.x : E.y;
+              if (me != v) continue;
+              const int val = (other << 2) | E.z;
+              if (E.z == 0) nbr[o0++] = val;
+              else if (E.z == 1) nbr[o1++] = val;
+              else if (E.z == 2) nbr[o2++] = val;
+              else nbr[o3++] = val;
+            }
           }
         }
       }
+
     }
     __syncthreads();
-    // which bond types occur in the tile (uniform loop, smem broadcast)
+    // which bond types occur in the tile (block-wide OR per type)
     int present = 0;
-    for (int i = 0; i < ne; ++i) present |= 1 << ed[i].z;
+    for (int b = 0; b < p.n_bonds; ++b) {
+      int mine = 0;
+      for (int i = tid; i < ne; i += kMpnnThreads) mine |= (ed[i].z == b);
+      if (__syncthreads_or(mine)) present |= 1 << b;
+    }
     // segments: 0 = U . h, 1..4 = W_b . s_b for bond types present
     int seg_list[5];
     int nseg = 0;
@@ -314,11 +366,21 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
 
     int wi = 0;   // weight buffer in use
     load_matrix_async(Wbuf[wi], p.u, tid);
+#ifdef MX_MPNN_PROF
+    long long tp1 = clock64();
+    c_setup += tp1 - tp0;
+#endif
     for (int step = 0; step < p.T; ++step) {
       bool s_ready = false;
       for (int si = 0; si < nseg; ++si) {
         const int seg = seg_list[si];
-        if (seg > 0 && !s_ready) build_s(sm, nbr_off, nbr, na, seg - 1, tid);
+#ifdef MX_MPNN_PROF
+        long long tb0 = clock64();
+#endif
+        if (seg > 0 && !s_ready) build_s(sm, off4, nbr, na, seg - 1, tid);
+#ifdef MX_MPNN_PROF
+        c_build += clock64() - tb0;
+#endif
         s_ready = false;
         cp_async_wait_all();
         fence_proxy_async();                   // S / H / W writes -> tensor-core reads
@@ -328,6 +390,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const uint16_t* nxt = nullptr;
         if (si + 1 < nseg) nxt = p.w_b + (size_t)(seg_list[si + 1] - 1) * kF * kF;
         else if (step + 1 < p.T) nxt = p.u;
+        else nxt = p.w1;   // readout weights, prefetched under the last MMA
         if (tid == 0) {
           tc_fence_after();
           const uint32_t a_hi = seg > 0 ? Shi : Hhi, a_lo = seg > 0 ? Slo : Hlo;
@@ -344,23 +407,29 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         if (nxt) load_matrix_async(Wbuf[wi ^ 1], nxt, tid);
         // the U.h contraction does not read S: build the next neighbour sum under it
         if (seg == 0 && si + 1 < nseg) {
-          build_s(sm, nbr_off, nbr, na, seg_list[si + 1] - 1, tid);
+          build_s(sm, off4, nbr, na, seg_list[si + 1] - 1, tid);
           s_ready = true;
         }
+#ifdef MX_MPNN_PROF
+        long long tm0 = clock64();
+#endif
         while (!mbar_try_wait_sleep(mma_bar, mma_phase, 1000)) {
         }
+#ifdef MX_MPNN_PROF
+        c_mma += clock64() - tm0;
+#endif
         mma_phase ^= 1;
         wi ^= 1;
       }
       // epilogue: h = ReLU(acc + c) -> hi/lo operand (padded rows stay 0).
-      // warp w: TMEM lanes 32(w%4).. (= atom rows), columns 64(w/4)..+63
+      // warp w: TMEM lanes 32(w%4).. (= atom rows), columns kEpiCols*(w/4)..
       tc_fence_after();
       {
         const int row = 32 * (warp & 3) + lane;
-        const int c0 = 64 * (warp >> 2);
+        const int c0 = kEpiCols * (warp >> 2);
         const uint32_t taddr = tmem + ((uint32_t)(32 * (warp & 3)) << 16) + (uint32_t)c0;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < kEpiCols / 16; ++q) {
           float v[16];
           tmem_ld16(taddr + 16 * q, v);
 #pragma unroll
@@ -379,18 +448,20 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       tc_fence_before();
       __syncthreads();
     }
+#ifdef MX_MPNN_PROF
+    long long tp2 = clock64();
+    c_steps += tp2 - tp1;
+#endif
     // readout: r_m = sum_v h_v (atom order); z_m = ReLU(W1 r_m + c1); y_m = w2 . z_m + c2,
     // W1 staged (swizzled) in a free weight buffer, molecules in batches of kReadoutMols
     cp_async_wait_all();
     __syncthreads();
-    load_matrix_async(Wbuf[0], p.w1, tid);
-    cp_async_wait_all();
-    __syncthreads();
+    const int offW1 = wi ? kOffW1 : kOffW0;   // buffer the last segment prefetched W1 into
     for (int mb = m0; mb < m1; mb += kReadoutMols) {
       const int nm = min(kReadoutMols, m1 - mb);
       for (int i = tid; i < nm * kF; i += kMpnnThreads) {
         const int mm = i / kF, f = i - mm * kF;
-        const int ab = p.atom_off[mb + mm] - a0, ae = p.atom_off[mb + mm + 1] - a0;
+        const int ab = moff[mb + mm - m0], ae = moff[mb + mm + 1 - m0];
         float t = 0.f;
         for (int v = ab; v < ae; ++v) {
           const uint32_t off = elem_off(v, f);
@@ -405,7 +476,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const float* r = rz + mm * 2 * kF;
         float t = bf16_bits_to_f32(p.c1[f]);
         for (int k = 0; k < kF; k += 8) {
-          const uint4 wv = *reinterpret_cast<const uint4*>(sm + kOffW0 + chunk_off(f, k >> 3));
+          const uint4 wv = *reinterpret_cast<const uint4*>(sm + offW1 + chunk_off(f, k >> 3));
           float wf[8];
           unpack8(wv, wf);
 #pragma unroll
@@ -427,7 +498,15 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       }
       __syncthreads();
     }
+#ifdef MX_MPNN_PROF
+    c_read += clock64() - tp2;
+#endif
   }
+#ifdef MX_MPNN_PROF
+  if (tid == 0 && blockIdx.x == 0)
+    printf("mpnn prof cta0: setup %lld steps %lld (build_s %lld, mma-wait %lld) readout %lld cycles\n",
+           c_setup, c_steps, c_build, c_mma, c_read);
+#endif
   tc_fence_before();
   __syncthreads();
   if (warp == 0) {
