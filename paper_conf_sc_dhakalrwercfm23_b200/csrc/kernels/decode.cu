@@ -35,8 +35,14 @@ int decode_prof_buckets() {
 #endif
 }
 
-int decode_fuse_attention(int B, int H, int hd) {
-  return (B < kTcMinBatch && B * H * hd <= 1024) ? 1 : 0;
+#ifndef MX_FUSE_MAX_CTAS
+#define MX_FUSE_MAX_CTAS 100000
+#endif
+// Fused attention (every CTA computes all heads inside the O phase) saves a
+// grid barrier per layer but replicates the K/V reads over the grid: used for
+// small attention on grids of at most MX_FUSE_MAX_CTAS CTAs.
+int decode_fuse_attention(int B, int H, int hd, int n_ctas) {
+  return (B < kTcMinBatch && B * H * hd <= 1024 && n_ctas <= MX_FUSE_MAX_CTAS) ? 1 : 0;
 }
 
 uint64_t decode_barriers(int L, int P, int G, int fuse_att) {

@@ -97,8 +97,8 @@ struct DecodeParams {
   unsigned long long done_tag;
 };
 
-// 1 if every CTA computes the whole attention itself (B*H*hd <= 1024).
-int decode_fuse_attention(int B, int H, int hd);
+// 1 if every CTA computes the whole attention itself (B*H*hd <= 1024, grid small enough).
+int decode_fuse_attention(int B, int H, int hd, int n_ctas);
 // 1 if this build records the per-CTA cycle buckets (-DMX_PROF_BUCKETS).
 int decode_prof_buckets();
 // Number of grid barriers one decode launch performs (host bookkeeping of bar_base).

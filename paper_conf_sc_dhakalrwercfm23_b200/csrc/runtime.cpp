@@ -714,7 +714,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.G = t->G;
     k.eps = c.rms_eps;
     k.n_ctas = e->n_ctas;
-    k.fuse_att = mxk::decode_fuse_attention(k.B, k.H, k.hd);
+    k.fuse_att = mxk::decode_fuse_attention(k.B, k.H, k.hd, k.n_ctas);
     const uint16_t* wb = reinterpret_cast<const uint16_t*>(fi->weights);
     k.w_layers = wb;
     k.layer_stride = fi->layer_stride;
