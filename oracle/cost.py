@@ -67,3 +67,9 @@ def decode_default_cost(cfg, batch, prompt_len, gen_len) -> int:
 
 def mpnn_default_cost(task: dict, F: int, T: int) -> int:
     return ceil_div(mpnn_task_flops(task, F, T), 75000)
+
+
+def mpnn_train_default_cost(task: dict, F: int, T: int) -> int:
+    """Placement cost of one emulator training step (N4, reading R10): forward
+    plus backward ~ 3x the forward contractions, same 75 TFLOP/s unit as C5."""
+    return ceil_div(3 * mpnn_task_flops(task, F, T), 75000)

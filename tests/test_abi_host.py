@@ -11,9 +11,9 @@ from hypothesis import given, settings, strategies as st
 
 from paper_conf_sc_dhakalrwercfm23_b200 import mx
 from oracle import sched as S
-from oracle.cost import decode_default_cost, mpnn_default_cost
+from oracle.cost import decode_default_cost, mpnn_default_cost, mpnn_train_default_cost
 from workloads.configs import TINY, GPT2S, LLAMA7B, MPNN
-from workloads.inputs import molecules, prompt_tokens
+from workloads.inputs import molecules, prompt_tokens, ip_targets
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -102,6 +102,31 @@ def test_default_cost_matches_oracle():
     desc = mx.mpnn_desc(MPNN, 64, 64 * 32, 64 * 64)
     t = mx.mpnn_task(1, mol)
     assert mx.task_default_cost(desc, t) == mpnn_default_cost(mol, MPNN.hidden, MPNN.steps)
+
+
+def test_training_and_shared_weight_descriptors_host_side():
+    """N4 cost rule (3x forward flops) and descriptor validation (N3/N4) are
+    pure host logic in libmx.so (no GPU needed)."""
+    mol = molecules(6, 24)
+    tdesc = mx.mpnn_train_desc(MPNN, 32, 32 * 32, 32 * 64)
+    t = mx.mpnn_train_task(1, mol, ip_targets(6, 24), 0.1)
+    assert mx.task_default_cost(tdesc, t) == mpnn_train_default_cost(mol, MPNN.hidden, MPNN.steps)
+    # a training step without targets is rejected
+    t.desc.targets = None
+    with pytest.raises(mx.MxError) as e:
+        mx.task_default_cost(tdesc, t)
+    assert e.value.code == mx.MX_EINVAL
+    # training state is per instance: shared weights are rejected for it
+    tdesc.flags = mx.MX_FN_SHARED_WEIGHTS
+    with pytest.raises(mx.MxError):
+        mx.task_default_cost(tdesc, mx.mpnn_train_task(1, mol, ip_targets(6, 24), 0.1))
+    # shared weights are accepted for inference functions, unknown flags are not
+    sdesc = mx.decode_desc(TINY, shared_weights=True)
+    td = mx.decode_task(1, prompt_tokens(1, 1, 8, TINY.vocab), 4)
+    assert mx.task_default_cost(sdesc, td) == decode_default_cost(TINY, 1, 8, 4)
+    sdesc.flags = 0x80
+    with pytest.raises(mx.MxError):
+        mx.task_default_cost(sdesc, td)
 
 
 def test_task_validation_rejects_bad_inputs():
