@@ -556,6 +556,105 @@ __device__ __forceinline__ void batched_loop(int n, int tid, int stride, Load lo
   }
 }
 
+// Tensor-core path (B >= kTcMinBatch) phase input from global fp32 activations
+// (x, o or a; RMSNorm'd where the phase has a gain): float4 loads (row widths
+// are multiples of 8) with kV4 loads in flight per thread, stored as the bf16
+// hi/lo operand. At batch 8 a K segment is 8 x ~1400 floats, so the scalar
+// 4-deep loop took ~8 L2 round trips per segment; this takes 2.
+constexpr int kV4 = 4;
+
+template <int B>
+__device__ __forceinline__ void stage_vec_tc(const DecodeParams& p, const Smem& sm,
+                                             const Phase& ph, const float* src,
+                                             const uint16_t* gain, int tid_c) {
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int K = ph.K, KP = ph.KP, k0 = ph.k0, KF = ph.ldw;
+  const int KP4 = KP >> 2, n4 = B * KP4;
+  if (gain && ph.seg == 0) {
+    // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt):
+    // per-thread partials, warp shuffle trees, fixed-order sum over warps; the
+    // scale is kept in smem for later K segments.
+    float acc[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) acc[b] = 0.f;
+    const int KF4 = KF >> 2, nf4 = B * KF4;
+    for (int base = tid_c; base < nf4; base += kV4 * kNCT) {
+      float4 v[kV4];
+#pragma unroll
+      for (int u = 0; u < kV4; ++u) {
+        const int i4 = base + u * kNCT;
+        if (i4 < nf4) {
+          const int b = i4 / KF4;
+          v[u] = *reinterpret_cast<const float4*>(src + (size_t)b * KF + ((i4 - b * KF4) << 2));
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < kV4; ++u) {
+        const int i4 = base + u * kNCT;
+        if (i4 < nf4) {
+          const int bi = i4 / KF4;
+          const float q = fmaf(v[u].x, v[u].x, fmaf(v[u].y, v[u].y, fmaf(v[u].z, v[u].z, v[u].w * v[u].w)));
+#pragma unroll
+          for (int b = 0; b < B; ++b)
+            if (b == bi) acc[b] += q;
+        }
+      }
+    }
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const float t = warp_sum(acc[b]);
+      if (lane == 0) sm.wsum[warp * 8 + b] = t;
+    }
+    named_bar_sync(1, kNCT);
+    if (tid_c < B) {
+      float t = 0.f;
+      for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + tid_c];
+      sm.inv[tid_c] = 1.0f / sqrtf(t / (float)KF + p.eps);
+    }
+    named_bar_sync(1, kNCT);
+  }
+  uint16_t* xh = reinterpret_cast<uint16_t*>(sm.xin);
+  uint16_t* xl = xh + B * (KP + 8);
+  for (int base = tid_c; base < n4; base += kV4 * kNCT) {
+    float4 v[kV4];
+#pragma unroll
+    for (int u = 0; u < kV4; ++u) {
+      const int i4 = base + u * kNCT;
+      if (i4 < n4) {
+        const int b = i4 / KP4, kk = (i4 - b * KP4) << 2;
+        v[u] = (kk < K) ? *reinterpret_cast<const float4*>(src + (size_t)b * KF + k0 + kk)
+                        : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kV4; ++u) {
+      const int i4 = base + u * kNCT;
+      if (i4 >= n4) continue;
+      const int b = i4 / KP4, kk = (i4 - b * KP4) << 2;
+      float f[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
+      if (gain && kk < K) {
+        const uint2 g = *reinterpret_cast<const uint2*>(gain + k0 + kk);
+        const float ib = sm.inv[b];
+        f[0] = f[0] * ib * bf16_bits_to_f32(g.x & 0xffffu);
+        f[1] = f[1] * ib * bf16_bits_to_f32(g.x >> 16);
+        f[2] = f[2] * ib * bf16_bits_to_f32(g.y & 0xffffu);
+        f[3] = f[3] * ib * bf16_bits_to_f32(g.y >> 16);
+      }
+      uint16_t h[4], l[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        h[j] = f32_to_bf16_rne(f[j]);
+        l[j] = f32_to_bf16_rne(f[j] - bf16_bits_to_f32(h[j]));
+      }
+      *reinterpret_cast<uint2*>(xh + b * (KP + 8) + kk) =
+          make_uint2(h[0] | ((uint32_t)h[1] << 16), h[2] | ((uint32_t)h[3] << 16));
+      *reinterpret_cast<uint2*>(xl + b * (KP + 8) + kk) =
+          make_uint2(l[0] | ((uint32_t)l[1] << 16), l[2] | ((uint32_t)l[3] << 16));
+    }
+  }
+  named_bar_sync(1, kNCT);
+}
+
 template <int B>
 __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                             int s, int tid_c) {
@@ -611,6 +710,12 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
     if (kind == PH_QKV) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gattn;
     if (kind == PH_GU) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gmlp;
     if (kind == PH_LM) gain = p.g_final;
+  }
+  if constexpr (B >= kTcMinBatch) {
+    if (!emb) {
+      stage_vec_tc<B>(p, sm, ph, src, gain, tid_c);
+      return;
+    }
   }
   // Inputs are read once into registers (up to kRegVals per thread), then the
   // RMSNorm scale is applied on the way into the lane-permuted smem layout.
