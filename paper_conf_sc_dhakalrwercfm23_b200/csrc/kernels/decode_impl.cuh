@@ -21,7 +21,8 @@
 //    bulk copies (cp.async.bulk) into a shared-memory ring of 32 KB stages
 //    guarded by mbarriers. The weight stream is static, so the producer runs
 //    ahead ACROSS phase barriers.
-//  * 12 decoupled consumer warps: a work unit is (output row, <= 1024-column
+//  * 11 decoupled consumer warps (12 warps per CTA = 3 per SM sub-partition, so
+//    the 168-register budget holds the GEMV without spills): a work unit is (output row, <= 1024-column
 //    group); each lane owns 8 consecutive columns of each 256-column chunk
 //    (one 16-byte smem load), the activations are staged in a lane-permuted
 //    layout so both 16-byte activation loads are bank-conflict free, and each
@@ -86,9 +87,10 @@ constexpr int kCPG = MX_CPG;                // 256-column chunks per GEMV work u
 // (kacc + partial). Segment widths depend only on the shape, so results stay
 // independent of the partition size.
 constexpr int kTcRows = 8;   // weight rows per tensor-core tile (the n of mma.m16n8k16)
-// kTcGroups tensor-core tiles are in progress at once.
+// kTcGroups tensor-core tiles are in progress at once (consumer warps beyond
+// kTcGroups * kTcSplit only observe and release the stages).
 constexpr int kTcGroups = kConsumerWarps / kTcSplit;
-static_assert(kConsumerWarps % kTcSplit == 0, "tensor-core warp groups must tile the consumers");
+static_assert(kTcGroups >= 1, "tensor-core split wider than the consumer warps");
 
 struct Phase {
   int kind, layer, R, K, KP, NC, NG, TR;
@@ -719,7 +721,10 @@ __device__ __forceinline__ void stage_input(const DecodeParams& p, const Smem& s
   }
   // Inputs are read once into registers (up to kRegVals per thread), then the
   // RMSNorm scale is applied on the way into the lane-permuted smem layout.
-  constexpr int kRegVals = 8;
+#ifndef MX_REG_VALS
+#define MX_REG_VALS 8
+#endif
+  constexpr int kRegVals = MX_REG_VALS;
   const bool in_regs = (B == 1) && (ph.nseg == 1) && (KP <= kRegVals * kNCT);
   float rv[kRegVals];
   auto load_in = [&](int b, int col) -> float {

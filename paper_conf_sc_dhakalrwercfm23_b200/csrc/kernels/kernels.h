@@ -10,7 +10,7 @@ namespace mxk {
 #define MX_STAGE_KB 32
 #endif
 #ifndef MX_CONSUMER_WARPS
-#define MX_CONSUMER_WARPS 12
+#define MX_CONSUMER_WARPS 11
 #endif
 #ifndef MX_MAX_STAGES
 #define MX_MAX_STAGES 6
@@ -41,7 +41,7 @@ MX_HD constexpr int decode_seg_cols(int B) { return (kXinSegBytes / (B * 4)) & ~
 #endif
 constexpr int kTcMinBatch = MX_TC_MIN_BATCH;
 #ifndef MX_TC_SPLIT
-#define MX_TC_SPLIT 4
+#define MX_TC_SPLIT 3
 #endif
 // A tensor-core tile (one stage) is consumed by kTcSplit warps that split its
 // K iterations.
