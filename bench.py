@@ -195,6 +195,22 @@ def gpu_arm(args, rank, world, local_rank, dist):
                           hbm_frac=sweep_tasks * bytes_task / s["span_s"] / (peak * 1e9)))
         for p in parts:
             mx.part_destroy(p)
+    # equal (MIG-like) layouts of the same N: STATIC (k-1) mod N placement
+    sweep_equal = []
+    for n in (args.sweep if args.sweep else []):
+        if n not in LAYOUTS_EQUAL or n == 1:
+            continue
+        parts = make_layout(mx, gpu, n, "equal")
+        load(parts)
+        run_batch(mx, fn, parts, min(sweep_tasks, 2 * len(parts)), True, prompts)   # warm
+        res, _ = run_batch(mx, fn, parts, sweep_tasks, True, prompts)
+        s = summarize(res, 1)
+        sweep_equal.append(dict(partitions=n, sms=LAYOUTS_EQUAL[n], tasks=sweep_tasks,
+                                tasks_per_s=sweep_tasks / s["span_s"], p50_ms=s["p50_ms"],
+                                p99_ms=s["p99_ms"],
+                                hbm_frac=sweep_tasks * bytes_task / s["span_s"] / (peak * 1e9)))
+        for p in parts:
+            mx.part_destroy(p)
     if args.layout == "auto":
         n_main = max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 14
     else:
@@ -288,6 +304,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
         "gen_tok_per_s": round(value * G_LEN, 1),
         "hbm_frac": round(achieved_gbs / peak, 4),
         "partitions_sweep": sweep,
+        "partitions_sweep_equal": sweep_equal,
         "roofline": {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak,
                      "unit": "GB/s", "frac": round(achieved_gbs / peak, 4), "traffic": traffic,
                      "kernel": "decode_kernel (persistent megakernel, all partitions together)",
