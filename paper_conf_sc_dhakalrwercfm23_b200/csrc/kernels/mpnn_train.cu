@@ -44,7 +44,8 @@ constexpr int kOffZ = kOffR + kF;                   // float [kF] a (pre-activat
 constexpr int kOffDA = kOffZ + kF;                  // float [kF] da
 constexpr int kOffDR = kOffDA + kF;                 // float [kF] dr
 constexpr int kOffRed = kOffDR + kF;                // float [16]
-constexpr int kTrainSmem = (kOffRed + 16) * 4;
+constexpr int kOffOff4 = kOffRed + 16;              // int [kA][5]: per-bond-type neighbour ranges
+constexpr int kTrainSmem = (kOffOff4 + kA * 5) * 4;
 // setup-only aliases inside the S buffer (before the first neighbour gather)
 constexpr int kOffEdges = kOffS;                    // int4 [kTE]
 constexpr int kOffMolE = kOffS + 4 * kTE;           // int2 [kA]
@@ -143,17 +144,29 @@ __device__ void gemm_grad(float* __restrict__ G, const float* Z, const float* Y,
     for (int j = 0; j < 8; ++j) G[(ta + 16 * i) * kF + tb + 16 * j] += acc.v[i][j];
 }
 
-// S[k][v] = sum over (u, b') in N(v) with b' == b of X[k][u] (neighbour-list order).
-__device__ void gather(float* S, const float* X, const int* nbr_off, const int* nbr, int na, int b,
+// S[k][v] = sum over the type-b neighbours u of v of X[k][u] (edge order). A
+// thread owns one atom v and half the features: its neighbour list is read
+// once (bucketed by bond type, off4[v][b] .. off4[v][b+1]) and reused for
+// every feature.
+constexpr int kGatherRegs = 8;
+__device__ void gather(float* S, const float* X, const int* off4, const int* nbr, int na, int b,
                        int tid) {
-  for (int i = tid; i < kF * kA; i += kThreads) {
-    const int k = i / kA, v = i - k * kA;
+  const int v = tid % kA, k0 = tid / kA;
+  int u[kGatherRegs];
+  int q0 = 0, q1 = 0;
+  if (v < na) {
+    q0 = off4[v * 5 + b];
+    q1 = off4[v * 5 + b + 1];
+  }
+  const int c = q1 - q0;
+#pragma unroll
+  for (int q = 0; q < kGatherRegs; ++q) u[q] = (q < c) ? (nbr[q0 + q] >> 2) : 0;
+  for (int k = k0; k < kF; k += kThreads / kA) {
     float t = 0.f;
-    if (v < na)
-      for (int q = nbr_off[v]; q < nbr_off[v + 1]; ++q) {
-        const int nb = nbr[q];
-        if ((nb & 3) == b) t += X[k * kS + (nb >> 2)];
-      }
+#pragma unroll
+    for (int q = 0; q < kGatherRegs; ++q)
+      if (q < c) t += X[k * kS + u[q]];
+    for (int q = q0 + kGatherRegs; q < q1; ++q) t += X[k * kS + (nbr[q] >> 2)];   // rare: deg > 8
     S[k * kS + v] = t;
   }
 }
@@ -183,6 +196,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   float* Wst = sm + kOffW;
   int* nbr_off = reinterpret_cast<int*>(sm + kOffNbrOff);
   int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
+  int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
   float* rr = sm + kOffR;
   float* aa = sm + kOffZ;
   float* da = sm + kOffDA;
@@ -254,11 +268,31 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         nbr_off[v] = pos;
         if (v == kA - 1) nbr_off[kA] = base + incl;
         if (v < na) {
+          // bucket v's neighbours by bond type, edge order inside a bucket
           const int2 er = mol_e[v];
+          int cnt = 0;   // 8-bit count per bond type
           for (int e = er.x; e < er.y; ++e) {
             const int4 Ev = ed[e];
-            if (Ev.x == v) nbr[pos++] = (Ev.y << 2) | Ev.z;
-            if (Ev.y == v) nbr[pos++] = (Ev.x << 2) | Ev.z;
+            cnt += ((Ev.x == v) + (Ev.y == v)) << (8 * Ev.z);
+          }
+          int o0 = pos, o1 = o0 + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255),
+              o3 = o2 + ((cnt >> 16) & 255);
+          off4[v * 5 + 0] = o0;
+          off4[v * 5 + 1] = o1;
+          off4[v * 5 + 2] = o2;
+          off4[v * 5 + 3] = o3;
+          off4[v * 5 + 4] = pos + deg;
+          for (int e = er.x; e < er.y; ++e) {
+            const int4 Ev = ed[e];
+            for (int side = 0; side < 2; ++side) {
+              const int me = side ? Ev.y : Ev.x, other = side ? Ev.x : Ev.y;
+              if (me != v) continue;
+              const int val = (other << 2) | Ev.z;
+              if (Ev.z == 0) nbr[o0++] = val;
+              else if (Ev.z == 1) nbr[o1++] = val;
+              else if (Ev.z == 2) nbr[o2++] = val;
+              else nbr[o3++] = val;
+            }
           }
         }
       }
@@ -280,7 +314,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       for (int b = 0; b < p.n_bonds; ++b) {
         if (!(present & (1 << b))) continue;
         __syncthreads();
-        gather(S, H, nbr_off, nbr, na, b, tid);
+        gather(S, H, off4, nbr, na, b, tid);
         gemm_xw_t(acc, S, Wb + (size_t)b * F * F, Wst, ta, tb, tid);   // syncs before reading S
       }
       __syncthreads();
@@ -373,11 +407,11 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       for (int b = 0; b < p.n_bonds; ++b) {
         if (!(present & (1 << b))) continue;
         __syncthreads();
-        gather(S, H, nbr_off, nbr, na, b, tid);                    // s_b(h^t)
+        gather(S, H, off4, nbr, na, b, tid);                    // s_b(h^t)
         __syncthreads();
         gemm_grad(G + p.off[1] + (size_t)b * F * F, D, S, ta, tb); // dW_b += dq^T s_b
         __syncthreads();
-        gather(S, D, nbr_off, nbr, na, b, tid);                    // sum of neighbours' dq
+        gather(S, D, off4, nbr, na, b, tid);                    // sum of neighbours' dq
         gemm_xw(acc, S, Wb + (size_t)b * F * F, Wst, ta, tb, tid); // dh += (.) W_b
       }
       __syncthreads();
