@@ -358,6 +358,83 @@ def cpu_baseline(args, n_tasks: int = 1):
                       f"fp64 NumPy oracle, weight generation excluded; {dt:.1f} s"}
 
 
+# --- D6: the CPU oracle on the box's host cores, per workload ----
+_CPU = {}
+
+
+def _cpu_decode_task(k):
+    from threadpoolctl import threadpool_limits
+    from oracle import decode as od
+    cfg, w, P, G = _CPU["decode"]
+    with threadpool_limits(1):
+        t0 = time.perf_counter()
+        od.greedy_task(cfg, w, prompt_tokens(k, 1, P, cfg.vocab), G)
+        return time.perf_counter() - t0
+
+
+def _cpu_mpnn_task(k):
+    from threadpoolctl import threadpool_limits
+    from oracle import mpnn as om
+    from workloads.configs import MPNN
+    from workloads.inputs import molecules
+    w, M = _CPU["mpnn"]
+    mol = molecules(k, M)
+    with threadpool_limits(1):
+        t0 = time.perf_counter()
+        om.mpnn_task(w, mol, MPNN.steps)
+        return time.perf_counter() - t0
+
+
+def cpu_suite():
+    """D6: one task per process, one BLAS thread per process, a pool of all host
+    cores; bounded samples of C1, C2, C4 (one wave each) and a 7B one-layer
+    decode step with BLAS on all cores (reported per layer-step: the full 7B
+    oracle would need ~27 GB of fp32 weights on the host; no extrapolation is
+    folded into the reported numbers)."""
+    import multiprocessing as mp
+    import platform
+    from oracle import decode as od
+    from workloads.configs import TINY, LLAMA7B, MPNN
+    from workloads.weights import decode_weights, mpnn_weights
+    cores = os.cpu_count() or 1
+    try:
+        model = [l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")][0]
+    except Exception:
+        model = platform.processor()
+    out = {"suite": "D6 cpu oracle", "host_cores": cores, "cpu_model": model, "rows": []}
+    ctx = mp.get_context("fork")
+    for name, cfg, P, G, n in (("C1 tiny decode", TINY, 8, 16, 4), ("C2 GPT-2s decode", GPT2S, P_LEN, G_LEN, cores)):
+        _CPU["decode"] = (cfg, decode_weights(cfg), P, G)
+        with ctx.Pool(min(n, cores)) as pool:
+            t0 = time.perf_counter()
+            per = pool.map(_cpu_decode_task, range(1, n + 1))
+            wall = time.perf_counter() - t0
+        out["rows"].append({"workload": name, "tasks": n, "procs": min(n, cores),
+                            "tasks_per_s": round(n / wall, 4), "task_s_median": round(float(np.median(per)), 3),
+                            "gen_tok_per_s": round(n * G / wall, 2)})
+    _CPU["mpnn"] = (mpnn_weights(MPNN), 1024)
+    n = cores
+    with ctx.Pool(n) as pool:
+        t0 = time.perf_counter()
+        per = pool.map(_cpu_mpnn_task, range(1, n + 1))
+        wall = time.perf_counter() - t0
+    out["rows"].append({"workload": "C4 MPNN inference (1024 molecules per task)", "tasks": n,
+                        "procs": n, "tasks_per_s": round(n / wall, 4),
+                        "task_s_median": round(float(np.median(per)), 3)})
+    from dataclasses import replace
+    cfg1 = replace(LLAMA7B.with_layers(1), vocab=1024)   # the layer's cost does not depend on V
+    w1 = decode_weights(cfg1)
+    st = od.DecodeState(cfg1, 64)
+    t0 = time.perf_counter()
+    for s in range(4):
+        od.decode_step(cfg1, w1, st, int(prompt_tokens(1, 1, 4, cfg1.vocab)[0, s]), s, want_logits=False)
+    per_layer_step = (time.perf_counter() - t0) / 4
+    out["rows"].append({"workload": "C3 7B decode, ONE layer (L=1 slice, vocab 1024), B=1, BLAS on all cores",
+                        "layer_step_ms": round(per_layer_step * 1e3, 2),
+                        "note": "a full 7B step is 32 such layers + the LM head; not measured"})
+    return out
+
+
 def reference_arm(args, rank, world):
     if rank != 0:
         return None
@@ -394,6 +471,8 @@ def main():
     ap.add_argument("--sweep", default="1,2,4,7,14,18,37",
                     help="comma list of partition counts for the pre-run sweep ('' = none)")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--cpu-suite", action="store_true",
+                    help="D6: time the CPU oracle per workload on the host cores and exit")
     ap.add_argument("--no-n3", dest="n3", action="store_false",
                     help="skip the shared-weights (N3) measurement of the chosen layout")
     args = ap.parse_args()
@@ -409,6 +488,10 @@ def main():
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         tdist.init_process_group("gloo", rank=rank, world_size=world)
         dist = tdist
+    if args.cpu_suite:
+        if rank == 0:
+            print(json.dumps(cpu_suite()), flush=True)
+        return
     if args.impl == "reference":
         out = reference_arm(args, rank, world)
     else:
