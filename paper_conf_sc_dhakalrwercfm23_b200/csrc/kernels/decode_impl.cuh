@@ -457,17 +457,34 @@ __device__ __forceinline__ void attend_hd(const DecodeParams& p, const Smem& sm,
     if (m > 0) load_block(m);
     const int j = m * KB + kslot;
     float dot = 0.f;
+    // q / k rows in smem are 16-byte aligned (kAttHd floats per row, kseg a
+    // multiple of 8): read them as float4 (a quarter of the LDS instructions)
     if (j < t) {
 #pragma unroll
       for (int i = 0; i < KV4; ++i) {
         float kf[8];
         unpack8(kr[i], kf);
-#pragma unroll
-        for (int q = 0; q < 8; ++q) dot = fmaf(qs[kseg + 8 * i + q], kf[q], dot);
+        const float4 qa = *reinterpret_cast<const float4*>(qs + kseg + 8 * i);
+        const float4 qb = *reinterpret_cast<const float4*>(qs + kseg + 8 * i + 4);
+        dot = fmaf(qa.x, kf[0], dot);
+        dot = fmaf(qa.y, kf[1], dot);
+        dot = fmaf(qa.z, kf[2], dot);
+        dot = fmaf(qa.w, kf[3], dot);
+        dot = fmaf(qb.x, kf[4], dot);
+        dot = fmaf(qb.y, kf[5], dot);
+        dot = fmaf(qb.z, kf[6], dot);
+        dot = fmaf(qb.w, kf[7], dot);
       }
     } else if (j == t) {
-#pragma unroll 8
-      for (int e = 0; e < KSEG; ++e) dot = fmaf(qs[kseg + e], ks[kseg + e], dot);
+#pragma unroll 4
+      for (int e = 0; e < KSEG; e += 4) {
+        const float4 qa = *reinterpret_cast<const float4*>(qs + kseg + e);
+        const float4 ka = *reinterpret_cast<const float4*>(ks + kseg + e);
+        dot = fmaf(qa.x, ka.x, dot);
+        dot = fmaf(qa.y, ka.y, dot);
+        dot = fmaf(qa.z, ka.z, dot);
+        dot = fmaf(qa.w, ka.w, dot);
+      }
     }
     if (LPK == 2) dot += __shfl_xor_sync(0xffffffffu, dot, 1);
     const float sc = (j <= t) ? dot / scale_div : -FLT_MAX;
