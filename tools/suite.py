@@ -201,8 +201,14 @@ def class_stats(res, kinds, mflops_mean, n_dec, n_mpnn):
         out[name] = s
     dec_bytes = n_dec * decode_task_bytes(GPT2S, 1, P_LEN, G_LEN)
     out["decode_hbm_frac"] = round(dec_bytes / sp / 1e9 / peak_gbs(), 4)
+    # share of the mixed run: MPNN flops over the whole makespan (decode dominates it)
     out["mpnn_tflops"] = round(n_mpnn * mflops_mean / sp / 1e12, 2)
     out["mpnn_tc_frac"] = round(out["mpnn_tflops"] / peak_bf16_tflops(), 4)
+    # the MPNN kernel itself: one task's flops over its median service time on its partition
+    if "mpnn" in out and out["mpnn"]["service_p50_ms"] > 0:
+        kt = mflops_mean / (out["mpnn"]["service_p50_ms"] * 1e-3) / 1e12
+        out["mpnn_kernel_tflops"] = round(kt, 2)
+        out["mpnn_kernel_tc_frac"] = round(kt / peak_bf16_tflops(), 4)
     out["tasks_per_s"] = round(len(res) / sp, 3)
     out["span_s"] = round(sp, 4)
     return out
