@@ -57,7 +57,7 @@ constexpr int kOffEdges = kOffW1 + kMatBytes;                  // int4 [kTileEdg
 constexpr int kOffMolE = kOffEdges + kTileEdges * 16;          // int2 [kTileAtoms]: edge range
 constexpr int kOffNbrOff = kOffMolE + kTileAtoms * 8;          // int [kTileAtoms+1] CSR offsets
 constexpr int kOffNbr = kOffNbrOff + (kTileAtoms + 4) * 4;     // int [2*kTileEdges]: (u<<2)|b
-constexpr int kReadoutMols = 4;                                // molecules per readout batch
+constexpr int kReadoutMols = 8;                                // molecules per readout batch (a tile holds ~6)
 constexpr int kOffR = kOffNbr + 2 * kTileEdges * 4;            // float [kReadoutMols][2][kF]: r, z
 constexpr int kOffC = kOffR + kReadoutMols * 2 * kF * 4;       // float [kF]: bias c
 constexpr int kOffRed = kOffC + kF * 4;                        // float [16]
@@ -463,6 +463,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const int mm = i / kF, f = i - mm * kF;
         const int ab = moff[mb + mm - m0], ae = moff[mb + mm + 1 - m0];
         float t = 0.f;
+#pragma unroll 4
         for (int v = ab; v < ae; ++v) {
           const uint32_t off = elem_off(v, f);
           t += bf16_bits_to_f32(*reinterpret_cast<const uint16_t*>(sm + kOffHhi + off)) +
@@ -475,12 +476,16 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const int mm = i / kF, f = i - mm * kF;
         const float* r = rz + mm * 2 * kF;
         float t = bf16_bits_to_f32(p.c1[f]);
+#pragma unroll 4
         for (int k = 0; k < kF; k += 8) {
           const uint4 wv = *reinterpret_cast<const uint4*>(sm + offW1 + chunk_off(f, k >> 3));
+          const float4 ra = *reinterpret_cast<const float4*>(r + k);
+          const float4 rb = *reinterpret_cast<const float4*>(r + k + 4);
+          const float rv[8] = {ra.x, ra.y, ra.z, ra.w, rb.x, rb.y, rb.z, rb.w};
           float wf[8];
           unpack8(wv, wf);
 #pragma unroll
-          for (int j = 0; j < 8; ++j) t = fmaf(wf[j], r[k + j], t);
+          for (int j = 0; j < 8; ++j) t = fmaf(wf[j], rv[j], t);
         }
         rz[mm * 2 * kF + kF + f] = fmaxf(t, 0.f);
       }
@@ -491,10 +496,9 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         float part = 0.f;
         for (int f = lane; f < kF; f += 32) part = fmaf(bf16_bits_to_f32(p.w2[f]), z[f], part);
         part = warp_sum(part);
-        if (lane == 0) {
-          p.out[mb + warp] = part + bf16_bits_to_f32(p.c2[0]);
-          __threadfence_system();   // ordered before the completion flag
-        }
+        // no per-molecule fence: the CTA's final __syncthreads + thread 0's
+        // __threadfence_system (cumulative) order these stores before the flag
+        if (lane == 0) p.out[mb + warp] = part + bf16_bits_to_f32(p.c2[0]);
       }
       __syncthreads();
     }
