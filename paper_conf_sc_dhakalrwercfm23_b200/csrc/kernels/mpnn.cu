@@ -218,10 +218,10 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
   int* moff = reinterpret_cast<int*>(sm + kOffMoff);
   int* eoff = reinterpret_cast<int*>(sm + kOffEoff);
-  uint8_t* typ = sm + kOffType;
   float* rz = reinterpret_cast<float*>(sm + kOffR);
   float* cvec = reinterpret_cast<float*>(sm + kOffC);
   float* red = reinterpret_cast<float*>(sm + kOffRed);
+  int* present_s = reinterpret_cast<int*>(sm + kOffRed) + 4;   // red[0..3] hold the degree scan
   uint64_t* mma_bar = reinterpret_cast<uint64_t*>(sm + kOffBar);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sm + kOffTmem);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -261,11 +261,22 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
     // tile-local molecule offsets, atom types and raw edges: independent loads,
     // one round trip
     const int nmt = m1 - m0;
+    if (tid == 0) *present_s = 0;   // previous tile's reads are many barriers back
     for (int j = tid; j <= nmt; j += kMpnnThreads) {
       moff[j] = p.atom_off[m0 + j] - a0;
       eoff[j] = p.edge_off[m0 + j] - e0;
     }
-    for (int i = tid; i < na; i += kMpnnThreads) typ[i] = p.atom_type[a0 + i];
+    // h0 = E_atom[type] (bf16-exact: hi = value, lo = 0); padded rows = 0. The
+    // type is read straight from global so these loads overlap the ones below.
+    for (int i = tid; i < kTileAtoms * kF / 8; i += kMpnnThreads) {
+      const int row = i >> 4, ch = i & 15;
+      uint4 hv = make_uint4(0, 0, 0, 0);
+      if (row < na)
+        hv = *reinterpret_cast<const uint4*>(p.e_atom + (size_t)p.atom_type[a0 + row] * kF + ch * 8);
+      const uint32_t off = chunk_off(row, ch);
+      *reinterpret_cast<uint4*>(sm + kOffHhi + off) = hv;
+      *reinterpret_cast<uint4*>(sm + kOffHlo + off) = make_uint4(0, 0, 0, 0);
+    }
     for (int i = tid; i < ne; i += kMpnnThreads) {
       const uint8_t* e = eb + (size_t)(e0 + i) * 6;
       ed[i] = make_int4((int)(int16_t)(e[0] | (e[1] << 8)), (int)(int16_t)(e[2] | (e[3] << 8)),
@@ -276,7 +287,9 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
     // search over the staged edge offsets)
     for (int j = tid; j < nmt; j += kMpnnThreads)
       for (int v = moff[j]; v < moff[j + 1]; ++v) mol_e[v] = make_int2(eoff[j], eoff[j + 1]);
+    int tmask = 0;   // bond types this thread's edges carry
     for (int i = tid; i < ne; i += kMpnnThreads) {
+      tmask |= 1 << ed[i].z;
       int lo = 0, hi = nmt - 1;
       while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
@@ -285,23 +298,21 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       ed[i].x += moff[lo];
       ed[i].y += moff[lo];
     }
-    // h0 = E_atom[type] (bf16-exact: hi = value, lo = 0); padded rows = 0
-    for (int i = tid; i < kTileAtoms * kF / 8; i += kMpnnThreads) {
-      const int row = i >> 4, ch = i & 15;
-      uint4 hv = make_uint4(0, 0, 0, 0);
-      if (row < na) hv = *reinterpret_cast<const uint4*>(p.e_atom + (size_t)typ[row] * kF + ch * 8);
-      const uint32_t off = chunk_off(row, ch);
-      *reinterpret_cast<uint4*>(sm + kOffHhi + off) = hv;
-      *reinterpret_cast<uint4*>(sm + kOffHlo + off) = make_uint4(0, 0, 0, 0);
-    }
+    tmask = __reduce_or_sync(0xffffffffu, tmask);
+    if (lane == 0 && tmask) atomicOr(present_s, tmask);   // read after the scan's barriers
     __syncthreads();
     // per-atom neighbour lists (CSR) in edge order: deterministic, built once per tile
     {
-      int deg = 0;
+      // one pass over the molecule's edges: 8-bit neighbour count per bond type
+      int deg = 0, cnt = 0;
       const int v = tid;
       if (v < kTileAtoms && v < na) {
         const int2 er = mol_e[v];
-        for (int e = er.x; e < er.y; ++e) deg += (ed[e].x == v) + (ed[e].y == v);
+        for (int e = er.x; e < er.y; ++e) {
+          const int4 E = ed[e];
+          cnt += ((E.x == v) + (E.y == v)) << (8 * E.z);
+        }
+        deg = (cnt & 255) + ((cnt >> 8) & 255) + ((cnt >> 16) & 255) + ((cnt >> 24) & 255);
       }
       // exclusive scan of degrees over the first 128 threads (4 warps)
       int incl = deg;
@@ -321,11 +332,6 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         if (v < na) {
           // bucket v's neighbours by bond type, edge order inside a bucket
           const int2 er = mol_e[v];
-          int cnt = 0;   // 8-bit count per bond type
-          for (int e = er.x; e < er.y; ++e) {
-            const int4 E = ed[e];
-            cnt += ((E.x == v) + (E.y == v)) << (8 * E.z);
-          }
           int o0 = pos, o1 = o0 + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255),
               o3 = o2 + ((cnt >> 16) & 255);
           off4[v * 5 + 0] = o0;
@@ -350,13 +356,8 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
 
     }
     __syncthreads();
-    // which bond types occur in the tile (block-wide OR per type)
-    int present = 0;
-    for (int b = 0; b < p.n_bonds; ++b) {
-      int mine = 0;
-      for (int i = tid; i < ne; i += kMpnnThreads) mine |= (ed[i].z == b);
-      if (__syncthreads_or(mine)) present |= 1 << b;
-    }
+    // which bond types occur in the tile (block-wide OR, gathered above)
+    const int present = *present_s & ((1 << p.n_bonds) - 1);
     // segments: 0 = U . h, 1..4 = W_b . s_b for bond types present
     int seg_list[5];
     int nseg = 0;
