@@ -249,7 +249,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   const uint32_t bar_s = smem_u32(mma_bar);
 
 #ifdef MX_MPNN_PROF
-  long long c_setup = 0, c_steps = 0, c_read = 0, c_build = 0, c_mma = 0;
+  long long c_setup = 0, c_steps = 0, c_read = 0, c_build = 0, c_mma = 0, c_ld = 0, c_nb = 0;
 #endif
   for (int tile = blockIdx.x; tile < p.n_tiles; tile += p.n_ctas) {
 #ifdef MX_MPNN_PROF
@@ -283,6 +283,10 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
                         (int)e[4], 0);
     }
     __syncthreads();
+#ifdef MX_MPNN_PROF
+    const long long tl = clock64();
+    c_ld += tl - tp0;
+#endif
     // atom -> its molecule's edge range; edges -> tile-local atom ids (binary
     // search over the staged edge offsets)
     for (int j = tid; j < nmt; j += kMpnnThreads)
@@ -330,32 +334,40 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         nbr_off[v] = pos;
         if (v == kTileAtoms - 1) nbr_off[kTileAtoms] = base + incl;
         if (v < na) {
-          // bucket v's neighbours by bond type, edge order inside a bucket
-          const int2 er = mol_e[v];
-          int o0 = pos, o1 = o0 + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255),
-              o3 = o2 + ((cnt >> 16) & 255);
-          off4[v * 5 + 0] = o0;
+          // v's neighbours bucketed by bond type: bucket b = off4[v][b] .. off4[v][b+1]
+          const int o1 = pos + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255);
+          off4[v * 5 + 0] = pos;
           off4[v * 5 + 1] = o1;
           off4[v * 5 + 2] = o2;
-          off4[v * 5 + 3] = o3;
+          off4[v * 5 + 3] = o2 + ((cnt >> 16) & 255);
           off4[v * 5 + 4] = pos + deg;
-          for (int e = er.x; e < er.y; ++e) {
-            const int4 E = ed[e];
-            for (int side = 0; side < 2; ++side) {
-              const int me = side ? E.y : E.x, other = side ? E.x : E.y;
-              if (me != v) continue;
-              const int val = (other << 2) | E.z;
-              if (E.z == 0) nbr[o0++] = val;
-              else if (E.z == 1) nbr[o1++] = val;
-              else if (E.z == 2) nbr[o2++] = val;
-              else nbr[o3++] = val;
-            }
-          }
         }
       }
-
     }
     __syncthreads();
+    // fill the buckets edge-parallel, edge order inside a bucket (the order a
+    // per-atom walk over the molecule's edges, side x then side y, produces):
+    // the rank of edge i's entry for endpoint `me` counts the earlier same-type
+    // edges of the molecule touching `me`, plus i's own side-x entry for side y.
+    for (int i = tid; i < ne; i += kMpnnThreads) {
+      const int4 E = ed[i];
+      const int eb0 = mol_e[E.x].x;
+      int rx = 0, ry = 0;
+      for (int e = eb0; e < i; ++e) {
+        const int4 F = ed[e];
+        if (F.z == E.z) {
+          rx += (F.x == E.x) + (F.y == E.x);
+          ry += (F.x == E.y) + (F.y == E.y);
+        }
+      }
+      ry += (E.x == E.y);
+      nbr[off4[E.x * 5 + E.z] + rx] = (E.y << 2) | E.z;
+      nbr[off4[E.y * 5 + E.z] + ry] = (E.x << 2) | E.z;
+    }
+    __syncthreads();
+#ifdef MX_MPNN_PROF
+    c_nb += clock64() - tl;   // remap + neighbour lists
+#endif
     // which bond types occur in the tile (block-wide OR, gathered above)
     const int present = *present_s & ((1 << p.n_bonds) - 1);
     // segments: 0 = U . h, 1..4 = W_b . s_b for bond types present
@@ -509,8 +521,8 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   }
 #ifdef MX_MPNN_PROF
   if (tid == 0 && blockIdx.x == 0)
-    printf("mpnn prof cta0: setup %lld steps %lld (build_s %lld, mma-wait %lld) readout %lld cycles\n",
-           c_setup, c_steps, c_build, c_mma, c_read);
+    printf("mpnn prof cta0: setup %lld (global loads %lld, remap+lists %lld) steps %lld (build_s %lld, mma-wait %lld) readout %lld cycles\n",
+           c_setup, c_ld, c_nb, c_steps, c_build, c_mma, c_read);
 #endif
   tc_fence_before();
   __syncthreads();
