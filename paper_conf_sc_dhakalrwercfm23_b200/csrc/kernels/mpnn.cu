@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
   const uint32_t Wbuf[2] = {sbase + kOffW0, sbase + kOffW1};
   int4* ed = reinterpret_cast<int4*>(sm + kOffEdges);
   int2* mol_e = reinterpret_cast<int2*>(sm + kOffMolE);
-  int* nbr_off = reinterpret_cast<int*>(sm + kOffNbrOff);
+  int* cnt_s = reinterpret_cast<int*>(sm + kOffNbrOff);   // per atom: 8-bit neighbour count per bond type
   int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
   int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
   int* moff = reinterpret_cast<int*>(sm + kOffMoff);
@@ -262,6 +262,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
     // one round trip
     const int nmt = m1 - m0;
     if (tid == 0) *present_s = 0;   // previous tile's reads are many barriers back
+    for (int i = tid; i < kTileAtoms; i += kMpnnThreads) cnt_s[i] = 0;
     for (int j = tid; j <= nmt; j += kMpnnThreads) {
       moff[j] = p.atom_off[m0 + j] - a0;
       eoff[j] = p.edge_off[m0 + j] - e0;
@@ -299,23 +300,24 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         const int mid = (lo + hi + 1) >> 1;
         if (eoff[mid] <= i) lo = mid; else hi = mid - 1;
       }
-      ed[i].x += moff[lo];
-      ed[i].y += moff[lo];
+      const int4 E = ed[i];
+      const int x = E.x + moff[lo], y = E.y + moff[lo];
+      ed[i].x = x;
+      ed[i].y = y;
+      // integer counts: the result does not depend on the atomics' order
+      atomicAdd(&cnt_s[x], 1 << (8 * E.z));
+      atomicAdd(&cnt_s[y], 1 << (8 * E.z));
     }
     tmask = __reduce_or_sync(0xffffffffu, tmask);
     if (lane == 0 && tmask) atomicOr(present_s, tmask);   // read after the scan's barriers
     __syncthreads();
     // per-atom neighbour lists (CSR) in edge order: deterministic, built once per tile
     {
-      // one pass over the molecule's edges: 8-bit neighbour count per bond type
+      // 8-bit neighbour count per bond type, gathered by the remap above
       int deg = 0, cnt = 0;
       const int v = tid;
       if (v < kTileAtoms && v < na) {
-        const int2 er = mol_e[v];
-        for (int e = er.x; e < er.y; ++e) {
-          const int4 E = ed[e];
-          cnt += ((E.x == v) + (E.y == v)) << (8 * E.z);
-        }
+        cnt = cnt_s[v];
         deg = (cnt & 255) + ((cnt >> 8) & 255) + ((cnt >> 16) & 255) + ((cnt >> 24) & 255);
       }
       // exclusive scan of degrees over the first 128 threads (4 warps)
@@ -331,8 +333,6 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
       for (int w = 0; w < warp && w < 4; ++w) base += __float_as_int(red[w]);
       if (v < kTileAtoms) {
         const int pos = base + incl - deg;
-        nbr_off[v] = pos;
-        if (v == kTileAtoms - 1) nbr_off[kTileAtoms] = base + incl;
         if (v < na) {
           // v's neighbours bucketed by bond type: bucket b = off4[v][b] .. off4[v][b+1]
           const int o1 = pos + (cnt & 255), o2 = o1 + ((cnt >> 8) & 255);
