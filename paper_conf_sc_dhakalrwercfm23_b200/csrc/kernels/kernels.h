@@ -151,6 +151,11 @@ struct MpnnParams {
 int mpnn_smem_bytes();
 // Greedy, deterministic packing of molecules into <=128-atom / <=512-bond tiles.
 int mpnn_pack_tiles(const int* atom_off, const int* edge_off, int n_mol, int* tile_off);
+// Same packing with a smaller atom cap per tile (<= 128): used to spread an
+// inference task over every CTA of the partition when the 128-atom packing
+// leaves part of the last round of tiles idle.
+int mpnn_pack_tiles_cap(const int* atom_off, const int* edge_off, int n_mol, int cap_atoms,
+                        int* tile_off);
 int launch_mpnn(const MpnnParams& p, void* stream);
 
 // IP-emulator training step (N4): tile forward/backward + SGD apply.

@@ -563,12 +563,18 @@ int mpnn_set_attrs(int device) { return set_max_smem(mpnn_kernel, mpnn_smem_byte
 // Deterministic greedy packing of molecules into tiles of <= 128 atoms and
 // <= 512 bonds (host side, runs at launch). Returns the number of tiles.
 int mpnn_pack_tiles(const int* atom_off, const int* edge_off, int n_mol, int* tile_off) {
+  return mpnn_pack_tiles_cap(atom_off, edge_off, n_mol, kTileAtoms, tile_off);
+}
+
+int mpnn_pack_tiles_cap(const int* atom_off, const int* edge_off, int n_mol, int cap_atoms,
+                        int* tile_off) {
+  if (cap_atoms > kTileAtoms || cap_atoms < 1) cap_atoms = kTileAtoms;
   int nt = 0;
   tile_off[0] = 0;
   int a = 0, e = 0;
   for (int m = 0; m < n_mol; ++m) {
     const int na = atom_off[m + 1] - atom_off[m], ne = edge_off[m + 1] - edge_off[m];
-    if ((a + na > kTileAtoms || e + ne > kTileEdges) && a > 0) {
+    if ((a + na > cap_atoms || e + ne > kTileEdges) && a > 0) {
       tile_off[++nt] = m;
       a = e = 0;
     }

@@ -778,7 +778,24 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     }
     // deterministic tile packing (host) -> device
     int* h5 = reinterpret_cast<int*>(h3 + align_up(t->n_atoms, 64) + align_up((size_t)t->n_edges * 6, 64));
-    const int n_tiles = mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
+    int n_tiles = mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
+    if (t->kind == MX_FN_MPNN && e->n_ctas > 0) {
+      // inference: a tile's time grows with its atoms, so fill the last round
+      // of CTAs with smaller tiles (same number of rounds, every CTA busy).
+      // Results are per molecule and do not depend on the tiling.
+      const int rounds = (n_tiles + e->n_ctas - 1) / e->n_ctas;
+      const int want = std::min(rounds * e->n_ctas, t->n_mol);
+      if (n_tiles < want) {
+        const int total = t->atom_off[t->n_mol] - t->atom_off[0];
+        int cap = std::max(1, (total + want - 1) / want);
+        int nt = 0;
+        for (; cap < 128; cap += 2) {
+          nt = mxk::mpnn_pack_tiles_cap(t->atom_off.data(), t->edge_off.data(), t->n_mol, cap, h5);
+          if (nt <= want) break;
+        }
+        n_tiles = cap < 128 ? nt : mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
+      }
+    }
     CU_TRY(drv().cuMemcpyHtoDAsync(s.tile_off, h5, (size_t)(n_tiles + 1) * 4, st));
     const mx_mpnn_cfg& m = d.mpnn;
     const uint16_t* wb = reinterpret_cast<const uint16_t*>(fi->weights);
