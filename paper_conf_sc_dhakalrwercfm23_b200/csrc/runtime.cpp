@@ -276,15 +276,17 @@ static void destroy_exec(Exec* e) {
   if (e->gctx) drv().cuGreenCtxDestroy(e->gctx);
 }
 
-// Unpartitioned exec (N1): a non-blocking stream of the primary context.
+// Unpartitioned exec (N1): a non-blocking stream of the GPU's whole-device
+// green context (every shared partition's stream lives in that one context,
+// like N processes' streams under the default MPS server).
 static int make_shared_exec(Gpu& gpu, int n_ctas, uint32_t epoch, std::unique_ptr<Exec>* out) {
   auto e = std::make_unique<Exec>();
   e->epoch = epoch;
   e->shared = true;
-  e->ctx = gpu.primary;
+  e->ctx = gpu.whole_ctx;
   e->n_ctas = n_ctas < gpu.sm_total ? n_ctas : gpu.sm_total;
-  CtxGuard g(gpu.primary);
-  CU_TRY(drv().cuStreamCreate(&e->stream, CU_STREAM_NON_BLOCKING));
+  CtxGuard g(gpu.whole_ctx);
+  CU_TRY(drv().cuGreenCtxStreamCreate(&e->stream, gpu.whole_gctx, CU_STREAM_NON_BLOCKING, 0));
   for (auto& lane : e->ev)
     for (auto& ev : lane)
       if (drv().cuEventCreate(&ev, CU_EVENT_DEFAULT) != CUDA_SUCCESS) {
@@ -1014,7 +1016,7 @@ static void dispatcher_main(Lib* L, Gpu* gpu) {
 static int calibrate_clock(Gpu& gpu) {
   CtxGuard cg(gpu.primary);
   CUstream st;
-  CU_TRY(drv().cuStreamCreate(&st, CU_STREAM_NON_BLOCKING));
+  CU_TRY(drv().cuGreenCtxStreamCreate(&st, gpu.whole_gctx, CU_STREAM_NON_BLOCKING, 0));
   CUdeviceptr dbuf = 0;
   Arena tmp;
   int rc = tmp.init(gpu.ordinal, 1 << 21, 1 << 21);
@@ -1093,6 +1095,12 @@ static int init_gpu(Gpu& gpu) {
       return MX_EDEVICE;
     }
   gpu.remainder = gpu.sm_total - gpu.n_groups * gpu.group_size;
+  {
+    CUdevResourceDesc wd;
+    CU_TRY(drv().cuDevResourceGenerateDesc(&wd, &gpu.whole, 1));
+    CU_TRY(drv().cuGreenCtxCreate(&gpu.whole_gctx, wd, gpu.dev, CU_GREEN_CTX_DEFAULT_STREAM));
+    CU_TRY(drv().cuCtxFromGreenCtx(&gpu.whole_ctx, gpu.whole_gctx));
+  }
   if (mxk::decode_set_attrs(gpu.dev) || mxk::mpnn_set_attrs(gpu.dev) ||
       mxk::mpnn_train_set_attrs(gpu.dev)) {
     set_error("setting kernel shared-memory attributes failed");
@@ -1238,7 +1246,10 @@ mx_status mx_shutdown(void) {
     if (g->wpool_ready) g->wpool.release();
     g->shared_w.clear();
   }
-  for (auto& g : L->gpus) drv().cuDevicePrimaryCtxRelease(g->dev);
+  for (auto& g : L->gpus) {
+    if (g->whole_gctx) drv().cuGreenCtxDestroy(g->whole_gctx);
+    drv().cuDevicePrimaryCtxRelease(g->dev);
+  }
   g_lib = nullptr;
   delete L;
   return MX_OK;

@@ -36,7 +36,7 @@ struct Exec {
   CUcontext ctx = nullptr;
   CUstream stream = nullptr;
   int n_ctas = 0;          // SMs provisioned (persistent grid size)
-  bool shared = false;     // primary-context stream, no SM restriction (N1); cooperative launches
+  bool shared = false;     // whole-device stream, no SM restriction (N1); cooperative launches
   uint32_t epoch = 0;
   CUevent ev[2][3] = {};   // per in-flight lane: kernel start, kernel end, done
   int inflight = 0;
@@ -157,6 +157,13 @@ struct Gpu {
   int sm_total = 0, n_groups = 0, group_size = 8, remainder = 0, cc_major = 0, cc_minor = 0;
   uint64_t mem_bytes = 0;
   CUdevResource whole{};
+  // A green context over the whole device: hosts the unpartitioned (N1) streams
+  // and the clock calibration, so that no kernel of the library ever runs in
+  // the primary context (an ncu launch list cannot follow a switch from a
+  // primary-context kernel to a green-context one: "Failed to prepare kernel",
+  // profiles/r2_ncu_green_ctx_probe.txt).
+  CUgreenCtx whole_gctx = nullptr;
+  CUcontext whole_ctx = nullptr;
   std::vector<CUdevResource> groups;
   int64_t clock_offset = 0;     // host_ns = device_ns + offset
   std::thread thr;
