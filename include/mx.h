@@ -42,7 +42,7 @@ enum {
   MX_EBUSY = -16,      /* resize shrink below used; destroy with pending work         */
   MX_ENODEV = -19,     /* gpu out of range, or device is not compute capability 10.x */
   MX_EINVAL = -22,     /* null/unknown handle, bad shape, sm_count <= 0 at create     */
-  MX_ENOSM = -28,      /* not enough free 8-SM groups (keeps sum of SMs <= device)    */
+  MX_ENOSM = -28,      /* not enough free SM groups (keeps sum of SMs <= device)      */
   MX_ETIMEDOUT = -110, /* fn_wait timed out; the task stays waitable                  */
   MX_ESTATE = -125     /* library not initialised (or already shut down)              */
 };
@@ -106,7 +106,9 @@ typedef struct {
   mx_mpnn_cfg mpnn;
 } mx_fn_desc;
 
-/* One bond of a molecule: atoms u, v are local indices within the molecule. */
+/* One bond of a molecule: atoms u, v are local indices within the molecule,
+ * u != v (a self-loop is MX_EINVAL at fn_submit, reading R12). The same pair
+ * may be listed more than once; each listing is a bond of C4's sum.         */
 typedef struct {
   int16_t u, v;
   uint8_t bond, pad;
@@ -149,10 +151,10 @@ typedef struct {
 } mx_result;
 
 typedef struct {
-  int32_t gpu, sm_count;  /* sm_count: SMs actually provisioned (8-SM groups, A20)     */
+  int32_t gpu, sm_count;  /* sm_count: SMs actually provisioned (whole SM groups, R8)  */
   int32_t n_ctas;         /* persistent grid size used for this partition              */
   int32_t whole;          /* 1 = the whole device (all groups + remainder)            */
-  uint64_t group_mask;    /* bit g = 8-SM group g of the device split                  */
+  uint64_t group_mask;    /* bit g = SM group g of the device split                    */
   uint64_t hbm_quota, hbm_used, hbm_peak;
   uint32_t epoch;
   uint32_t shared;        /* 1 = unpartitioned stream (part_create_shared, N1)        */
@@ -170,8 +172,12 @@ typedef struct {
 /* Initialise on every visible GPU of compute capability 10.x. Sets
  * CUDA_DEVICE_MAX_CONNECTIONS=32 if unset (only effective before the first
  * CUDA call of the process), retains each primary context, splits each
- * device's SMs once into 8-SM groups (cuDevSmResourceSplitByCount) and starts
- * one dispatcher thread per GPU. MX_ENODEV if no suitable GPU.             */
+ * device's SMs once into equal SM groups (cuDevSmResourceSplitByCount; on a
+ * B200 37 groups of 4 SMs, reading R8 in DESIGN.md; MX_SM_GROUP=8 selects the
+ * co-scheduling-aware 8-SM split), creates one whole-device green context
+ * (clock calibration, unpartitioned N1 streams: no library kernel runs in the
+ * primary context) and starts one dispatcher thread per GPU. MX_ENODEV if no
+ * suitable GPU.                                                            */
 mx_status mx_init(uint32_t flags);
 /* Same, restricted to the listed device ordinals (e.g. one per torchrun rank). */
 mx_status mx_init_devices(const int32_t* ordinals, int32_t n, uint32_t flags);
@@ -187,7 +193,7 @@ const char* mx_last_error(void);   /* thread-local detail of the last failure   
  * ------------------------------------------------------------------------- */
 
 /* Create a partition of `gpu` with at least `sm_count` SMs (rounded up to whole
- * 8-SM groups, lowest free groups first; sm_count >= the device's SM count asks
+ * SM groups, lowest free groups first; sm_count >= the device's SM count asks
  * for the whole device) and an HBM quota of `hbm_bytes` enforced by the
  * partition's allocator arena (A23: a capacity limit, not bandwidth or fault
  * isolation). Errors: MX_ENODEV, MX_EINVAL, MX_ENOSM, MX_ENOMEM (sum of quotas
@@ -195,7 +201,7 @@ const char* mx_last_error(void);   /* thread-local detail of the last failure   
 mx_status part_create(int32_t gpu, int32_t sm_count, uint64_t hbm_bytes, int32_t* out_part);
 /* Unpartitioned comparison mode (Table 1
  * and §5.2: time-sharing vs MPS vs MIG). The partition is a plain
- * stream of the primary context: it owns NO SM groups (not counted in the
+ * stream of the GPU's whole-device green context: it owns NO SM groups (not counted in the
  * 148-SM budget, I2), its kernels may run on any SM, and decode grids are
  * `n_ctas` CTAs launched cooperatively (all CTAs co-resident or none).
  *   n_ctas = SM count  -> every task wants the whole GPU: tasks of different
@@ -266,6 +272,12 @@ mx_status mx_probe_smids_concurrent(const int32_t* parts, int32_t n_parts, int32
 mx_status mx_decode_profile(int32_t part, uint64_t* out, int32_t n_words);
 /* Number of kernels this library launched since init (all GPUs).          */
 mx_status mx_launch_count(uint64_t* out);
+/* Fault-path test hook: the next task LAUNCHED on `part` runs normally but its
+ * kernel reports device error `code` (> 0) in its completion record, exactly
+ * as a bounded-wait timeout would (SURVEY.md §8(b) MX_EDEVICE row: "the task
+ * still completes exactly once, with this status"). The slot is reset before
+ * its next use. MX_EINVAL for an unknown partition or code <= 0.           */
+mx_status mx_debug_inject_error(int32_t part, int32_t code);
 
 /* ---------------------------------------------------------------------------
  * Host-only placement engine (no device needed): the same C++ object the

@@ -48,6 +48,15 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None,
     bdir = build_dir or BUILD
     os.makedirs(bdir, exist_ok=True)
     hdr_mtime = max(os.path.getmtime(h) for h in headers())
+    # objects are only reused when built with the same flags (a variant build
+    # with MX_DEFS must never leak its objects into the product library)
+    stamp = os.path.join(bdir, "flags.stamp")
+    flags = " ".join(ARCH + EXTRA_DEFS)
+    if not os.path.exists(stamp) or open(stamp).read() != flags:
+        force = True
+    lib_stamp = lib + ".flags"
+    if not os.path.exists(lib_stamp) or open(lib_stamp).read() != flags:
+        force = True
     objs, jobs = [], []
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "-I", CSRC,
               "-I", os.path.join(ROOT, "include")] + EXTRA_DEFS
@@ -86,6 +95,9 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None,
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)
             raise RuntimeError("link failed")
+    for path in (stamp, lib_stamp):
+        with open(path, "w") as f:
+            f.write(flags)
     return lib
 
 

@@ -1437,11 +1437,13 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     if (tid_c == 0) {
       const unsigned long long t_end = globaltimer();
       p.stamps[1] = t_end;
+      if (p.inject_err && !p.h_stamps) atomicExch(p.err, p.inject_err);
       if (p.h_stamps) {
         // every CTA passed the last grid barrier, so all outputs are final
         volatile unsigned long long* h = p.h_stamps;
         h[0] = p.stamps[0];
         h[1] = t_end;
+        if (p.inject_err) atomicExch(p.err, p.inject_err);   // fault-path test hook
         h[2] = (unsigned long long)(unsigned)ld_volatile_i32(p.err);
         __threadfence_system();
         h[3] = p.done_tag;

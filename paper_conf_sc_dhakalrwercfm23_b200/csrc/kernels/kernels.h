@@ -95,6 +95,7 @@ struct DecodeParams {
   // written last (after a system-scope fence) by CTA 0
   unsigned long long* h_stamps;
   unsigned long long done_tag;
+  int inject_err;            // test hook (mx_debug_inject_error): reported as the task's device error
 };
 
 // 1 if every CTA computes the whole attention itself (B*H*hd <= 1024, grid small enough).
@@ -147,6 +148,7 @@ struct MpnnParams {
   // finish; stamps[4] is the CTA-completion counter (reset by that CTA)
   unsigned long long* h_stamps;
   unsigned long long done_tag;
+  int inject_err;            // test hook (mx_debug_inject_error): reported as the task's device error
 };
 int mpnn_smem_bytes();
 // Greedy, deterministic packing of molecules into <=128-atom / <=512-bond tiles.
@@ -177,6 +179,7 @@ struct MpnnTrainParams {
   unsigned long long* stamps;
   unsigned long long* h_stamps;
   unsigned long long done_tag;
+  int inject_err;            // test hook (mx_debug_inject_error): reported as the task's device error
 };
 int mpnn_train_smem_bytes();
 uint64_t mpnn_train_tile_scratch_floats(int T);

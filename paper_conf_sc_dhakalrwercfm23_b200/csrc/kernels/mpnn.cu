@@ -542,7 +542,7 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         volatile unsigned long long* h = p.h_stamps;
         h[0] = st[0];
         h[1] = st[1];
-        h[2] = 0;
+        h[2] = (unsigned long long)(unsigned)p.inject_err;   // 0 unless the fault-path test hook is set
         p.stamps[4] = 0;
         __threadfence_system();
         h[3] = p.done_tag;

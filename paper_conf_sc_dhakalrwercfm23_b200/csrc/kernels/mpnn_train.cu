@@ -458,7 +458,7 @@ __global__ void __launch_bounds__(kThreads) mpnn_train_apply_kernel(MpnnTrainPar
       volatile unsigned long long* h = p.h_stamps;
       h[0] = st[0];
       h[1] = globaltimer();
-      h[2] = 0;
+      h[2] = (unsigned long long)(unsigned)p.inject_err;   // 0 unless the fault-path test hook is set
       p.stamps[4] = 0;
       __threadfence_system();
       h[3] = p.done_tag;

@@ -118,15 +118,14 @@ static uint64_t decode_task_bytes(const mx_decode_cfg& c, uint64_t B, uint64_t P
          B * kvpos * (S * (S + 1) / 2) + S * B * kvpos;
 }
 
-static uint64_t mpnn_mol_flops(int n, const uint8_t* edges6, int ne, uint64_t F, uint64_t T) {
-  std::set<std::pair<int, int>> pairs;
-  for (int i = 0; i < ne; ++i) {
-    const uint8_t* e = edges6 + (size_t)i * 6;
-    int u = (int16_t)(e[0] | (e[1] << 8)), v = (int16_t)(e[2] | (e[3] << 8)), b = e[4];
-    pairs.insert({u, b});
-    pairs.insert({v, b});
-  }
-  const uint64_t D = pairs.size(), edir = 2ull * ne, nn = (uint64_t)n;
+// D_ub = distinct (atom, incident bond type) pairs: one 32-bit atom mask per
+// bond type (molecules have <= 32 atoms, <= 4 bond types; validated first).
+static uint64_t mpnn_mol_flops(int n, const mx_bond* e, int ne, uint64_t F, uint64_t T) {
+  uint32_t mask[4] = {0, 0, 0, 0};
+  for (int i = 0; i < ne; ++i) mask[e[i].bond & 3] |= (1u << e[i].u) | (1u << e[i].v);
+  const uint64_t D = (uint64_t)(__builtin_popcount(mask[0]) + __builtin_popcount(mask[1]) +
+                                __builtin_popcount(mask[2]) + __builtin_popcount(mask[3]));
+  const uint64_t edir = 2ull * ne, nn = (uint64_t)n;
   return T * (2 * F * F * (nn + D) + edir * F + 2 * nn * F) + nn * F + 2 * F * F + 4 * F;
 }
 
@@ -236,6 +235,10 @@ static int validate_task(const mx_fn_desc& d, const mx_task_desc& t) {
         set_error("mpnn task: bond %d of molecule %d out of range", e, i);
         return MX_EINVAL;
       }
+      if (b.u == b.v) {   // reading R12: a bond joins two distinct atoms
+        set_error("mpnn task: bond %d of molecule %d is a self-loop", e, i);
+        return MX_EINVAL;
+      }
     }
   }
   for (int i = 0; i < t.n_atoms; ++i)
@@ -250,11 +253,10 @@ static uint64_t default_cost(const mx_fn_desc& d, const mx_task_desc& t) {
   if (d.kind == MX_FN_DECODE)
     return ceil_div(decode_task_bytes(d.dec, t.batch, t.prompt_len, t.gen_len), 8000);
   uint64_t fl = 0;
-  const uint8_t* eb = reinterpret_cast<const uint8_t*>(t.edges);
   for (int i = 0; i < t.n_mol; ++i) {
     const int n = t.atom_off[i + 1] - t.atom_off[i];
     const int ne = t.edge_off[i + 1] - t.edge_off[i];
-    fl += mpnn_mol_flops(n, eb + (size_t)t.edge_off[i] * 6, ne, (uint64_t)d.mpnn.hidden,
+    fl += mpnn_mol_flops(n, t.edges + t.edge_off[i], ne, (uint64_t)d.mpnn.hidden,
                          (uint64_t)d.mpnn.steps);
   }
   // training: forward + backward ~ 3x the forward contractions (N4)
@@ -509,29 +511,36 @@ static int alloc_decode_slot(Partition& p, FnInst& fi, Slot& s) {
   return MX_OK;
 }
 
+// Byte layout of a MPNN task's packed inputs (Task::blob, Slot::in_blob).
+static size_t mpnn_blob_layout(Task& t, bool train, int n_mol, int n_atoms, int n_edges) {
+  const size_t offs = align_up((uint64_t)(n_mol + 1) * 4, 64);
+  t.off_ao = 0;
+  t.off_eo = (uint32_t)offs;
+  t.off_tile = (uint32_t)(2 * offs);
+  t.off_tg = (uint32_t)(3 * offs);
+  t.off_at = (uint32_t)(t.off_tg + (train ? align_up((uint64_t)n_mol * 4, 64) : 0));
+  t.off_ed = (uint32_t)(t.off_at + align_up((uint64_t)n_atoms, 64));
+  return t.off_ed + align_up((uint64_t)n_edges * 6, 64);
+}
+
 static int alloc_mpnn_slot(Partition& p, FnInst& fi, Slot& s) {
   const mx_mpnn_cfg& m = fi.fn->desc.mpnn;
-  const uint64_t M = m.max_mols, NA = m.max_atoms, NE = std::max(1, m.max_edges);
+  const bool train = fi.fn->desc.kind == MX_FN_MPNN_TRAIN;
+  const uint64_t M = m.max_mols;
   int rc;
-  if ((rc = alloc_ptr(p, (M + 1) * 4, &s.atom_off))) return rc;
-  if ((rc = alloc_ptr(p, NA, &s.atom_type))) return rc;
-  if ((rc = alloc_ptr(p, (M + 1) * 4, &s.edge_off))) return rc;
-  if ((rc = alloc_ptr(p, NE * 6, &s.edges))) return rc;
-  if ((rc = alloc_ptr(p, M * 4, &s.out))) return rc;
-  if ((rc = alloc_ptr(p, (M + 1) * 4, &s.tile_off))) return rc;
+  Task probe;
+  s.h_in_bytes = mpnn_blob_layout(probe, train, m.max_mols, m.max_atoms, std::max(1, m.max_edges));
+  if ((rc = alloc_ptr(p, s.h_in_bytes, &s.in_blob))) return rc;
   if ((rc = alloc_ptr(p, 64, &s.stamps))) return rc;
   s.err = s.stamps + 16;
-  s.h_in_bytes = align_up((M + 1) * 4, 64) * 3 + align_up(NA, 64) + align_up(NE * 6, 64) + 64;
   s.h_out_bytes = M * 4;
-  if (fi.fn->desc.kind == MX_FN_MPNN_TRAIN) {
+  if (train) {
     // tiles hold >= 4 molecules (<= 32 atoms each) except the last
     const uint64_t tiles = (M + 3) / 4 + 1;
-    if ((rc = alloc_ptr(p, M * 4, &s.targets))) return rc;
     if ((rc = alloc_ptr(p, M * 4, &s.y))) return rc;
     if ((rc = alloc_ptr(p, tiles * fi.n_params * 4, &s.partials))) return rc;
     if ((rc = alloc_ptr(p, tiles * mxk::mpnn_train_tile_scratch_floats(m.steps) * 4, &s.hsave)))
       return rc;
-    s.h_in_bytes += align_up(M * 4, 64);
     s.h_out_bytes = (M + 1) * 4;
   }
   if ((rc = host_alloc(s.h_in_bytes, &s.h_in, &s.d_in))) return rc;
@@ -576,7 +585,31 @@ static int generate_weights(FnInst& fi, CUstream st, int nct) {
   return MX_OK;
 }
 
-// Caller holds p.load_mu. Synchronous cold start on the partition's stream.
+static void free_slot_host(Slot& s) {
+  if (s.h_in) drv().cuMemFreeHost(s.h_in);
+  if (s.h_out) drv().cuMemFreeHost(s.h_out);
+  if (s.h_stamps) drv().cuMemFreeHost(s.h_stamps);
+  s.h_in = s.h_out = nullptr;
+  s.h_stamps = nullptr;
+}
+
+// Drop one partition instance's reference to shared weights (N3); once no
+// instance on the GPU references any shared weights, the pool is unmapped.
+static void release_shared_ref(Gpu& gpu, int fn_id) {
+  std::lock_guard<std::mutex> wl(gpu.wpool_mu);
+  auto it = gpu.shared_w.find(fn_id);
+  if (it == gpu.shared_w.end()) return;
+  it->second.refs--;
+  for (auto& kv : gpu.shared_w)
+    if (kv.second.refs > 0) return;
+  if (gpu.wpool_ready) gpu.wpool.release();
+  gpu.wpool_ready = false;
+  gpu.shared_w.clear();
+}
+
+// Caller holds p.load_mu (part_resize / part_destroy take it too, so p.cur and
+// its stream stay fixed while the load runs). Synchronous cold start on the
+// partition's stream.
 static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
   auto it = p.insts.find(fn.id);
   if (it != p.insts.end() && it->second->loaded) {
@@ -640,25 +673,41 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
       if ((rc = alloc_ptr(p, (uint64_t)c.max_seq * c.head_dim * 4, &fi->rope))) return rc;
     }
   }
+  // from here on a failure releases the pinned host staging already allocated
+  // (arena bytes stay used: bump allocator; reported by part_query)
+  auto fail = [&](int code) {
+    for (Slot& s : fi->slots) free_slot_host(s);
+    if (fi->shared_weights) {
+      std::lock_guard<std::mutex> wl(gpu.wpool_mu);
+      gpu.shared_w[fn.id].refs--;
+    }
+    return code;
+  };
   for (Slot& s : fi->slots) {
     rc = (d.kind == MX_FN_DECODE) ? alloc_decode_slot(p, *fi, s) : alloc_mpnn_slot(p, *fi, s);
-    if (rc) return rc;   // arena bytes stay used (bump allocator); reported by part_query
+    if (rc) return fail(rc);
   }
-  if (!fi->shared_weights && (rc = generate_weights(*fi, st, nct))) return rc;
+  if (!fi->shared_weights && (rc = generate_weights(*fi, st, nct))) return fail(rc);
   if (d.kind == MX_FN_MPNN_TRAIN) {
     // fp32 training state, widened exactly from the seeded bf16 values (N4)
     if (mxk::launch_widen_bf16(reinterpret_cast<float*>(fi->params),
                                reinterpret_cast<const uint16_t*>(fi->weights), fi->n_params, nct,
                                st)) {
       set_error("parameter widening launch failed");
-      return MX_EDEVICE;
+      return fail(MX_EDEVICE);
     }
   }
   for (Slot& s : fi->slots) {
-    if (s.bar) CU_TRY(drv().cuMemsetD8Async(s.bar, 0, 64, st));
-    CU_TRY(drv().cuMemsetD8Async(s.stamps, 0, 64, st));
+    if ((s.bar && drv().cuMemsetD8Async(s.bar, 0, 64, st) != CUDA_SUCCESS) ||
+        drv().cuMemsetD8Async(s.stamps, 0, 64, st) != CUDA_SUCCESS) {
+      set_error("slot reset failed");
+      return fail(MX_EDEVICE);
+    }
   }
-  CU_TRY(drv().cuStreamSynchronize(st));
+  if (drv().cuStreamSynchronize(st) != CUDA_SUCCESS) {
+    set_error("cold start on partition %d failed on the device", p.id);
+    return fail(MX_EDEVICE);
+  }
   fi->loaded = true;
   *out = fi.get();
   p.insts[fn.id] = std::move(fi);
@@ -668,6 +717,35 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
 // ---------------------------------------------------------------------------
 // Dispatcher
 // ---------------------------------------------------------------------------
+
+// Inference tiling for a partition of n_ctas CTAs: the 128-atom next-fit
+// packing, unless its last round of tiles would leave CTAs idle — then the
+// smallest atom cap (start + 2k, < 128) whose packing has at most
+// rounds * n_ctas tiles, so every CTA of the last round gets a (smaller) tile.
+// Next-fit tile counts do not increase with the cap, so a binary search finds
+// the same cap as a linear scan. Results are per molecule and do not depend on
+// the tiling (tested bit-identical across partition sizes).
+static int balanced_tiles(const int* ao, const int* eo, int n_mol, int n_ctas, int* tile_off) {
+  const int nt = mxk::mpnn_pack_tiles(ao, eo, n_mol, tile_off);
+  if (n_ctas <= 0) return nt;
+  const int rounds = (nt + n_ctas - 1) / n_ctas;
+  const int want = std::min(rounds * n_ctas, n_mol);
+  if (nt >= want) return nt;
+  const int total = ao[n_mol] - ao[0];
+  const int start = std::max(1, (total + want - 1) / want);
+  const int K = start < 128 ? (128 - start + 1) / 2 : 0;
+  int lo = 0, hi = K;
+  while (lo < hi) {
+    const int mid = (lo + hi) / 2;
+    if (mxk::mpnn_pack_tiles_cap(ao, eo, n_mol, start + 2 * mid, tile_off) <= want)
+      hi = mid;
+    else
+      lo = mid + 1;
+  }
+  if (lo < K) return mxk::mpnn_pack_tiles_cap(ao, eo, n_mol, start + 2 * lo, tile_off);
+  return mxk::mpnn_pack_tiles(ao, eo, n_mol, tile_off);
+}
+
 static int launch_task(Gpu& gpu, Partition& p, Task* t) {
   Exec* e = p.cur.get();
   t->exec = e;
@@ -686,6 +764,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     s.need_reset = false;
   }
   const mx_fn_desc& d = fi->fn->desc;
+  const int inject = p.inject_err.exchange(0);
   // Completion: the kernel writes its results and a done tag into host-mapped
   // memory, so a task is ONE kernel launch in the stream with nothing queued
   // behind it (copies / event records after a kernel would block unrelated
@@ -743,6 +822,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.tokens = reinterpret_cast<int*>(s.d_out);
     k.h_stamps = reinterpret_cast<unsigned long long*>(s.d_stamps);
     k.done_tag = t->id;
+    k.inject_err = inject;
     k.logits = t->out_logits ? reinterpret_cast<float*>(s.logits) : nullptr;
     k.bar = reinterpret_cast<unsigned long long*>(s.bar);
     k.bar_base = s.bar_count;
@@ -762,43 +842,18 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
                                      s.logits, (size_t)t->G * t->B * c.vocab * 4, st));
     }
   } else {
-    // pack CSR inputs into pinned staging, one H2D per array
-    uint8_t* h = static_cast<uint8_t*>(s.h_in);
-    const size_t b_off = (size_t)(t->n_mol + 1) * 4;
-    memcpy(h, t->atom_off.data(), b_off);
-    CU_TRY(drv().cuMemcpyHtoDAsync(s.atom_off, h, b_off, st));
-    uint8_t* h2 = h + align_up(b_off, 64);
-    memcpy(h2, t->edge_off.data(), b_off);
-    CU_TRY(drv().cuMemcpyHtoDAsync(s.edge_off, h2, b_off, st));
-    uint8_t* h3 = h2 + align_up(b_off, 64);
-    memcpy(h3, t->atom_type.data(), t->n_atoms);
-    CU_TRY(drv().cuMemcpyHtoDAsync(s.atom_type, h3, t->n_atoms, st));
-    if (t->n_edges > 0) {
-      uint8_t* h4 = h3 + align_up(t->n_atoms, 64);
-      memcpy(h4, t->edges.data(), (size_t)t->n_edges * 6);
-      CU_TRY(drv().cuMemcpyHtoDAsync(s.edges, h4, (size_t)t->n_edges * 6, st));
+    // the inputs were packed at submit in their device image: one H2D copy
+    if (t->kind == MX_FN_MPNN && t->tile_ctas != e->n_ctas) {
+      // the partition was resized after submit: re-balance the tiles for its CTA count
+      const int* ao = reinterpret_cast<const int*>(t->blob.data() + t->off_ao);
+      const int* eo = reinterpret_cast<const int*>(t->blob.data() + t->off_eo);
+      t->n_tiles = balanced_tiles(ao, eo, t->n_mol, e->n_ctas,
+                                  reinterpret_cast<int*>(t->blob.data() + t->off_tile));
+      t->tile_ctas = e->n_ctas;
     }
-    // deterministic tile packing (host) -> device
-    int* h5 = reinterpret_cast<int*>(h3 + align_up(t->n_atoms, 64) + align_up((size_t)t->n_edges * 6, 64));
-    int n_tiles = mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
-    if (t->kind == MX_FN_MPNN && e->n_ctas > 0) {
-      // inference: a tile's time grows with its atoms, so fill the last round
-      // of CTAs with smaller tiles (same number of rounds, every CTA busy).
-      // Results are per molecule and do not depend on the tiling.
-      const int rounds = (n_tiles + e->n_ctas - 1) / e->n_ctas;
-      const int want = std::min(rounds * e->n_ctas, t->n_mol);
-      if (n_tiles < want) {
-        const int total = t->atom_off[t->n_mol] - t->atom_off[0];
-        int cap = std::max(1, (total + want - 1) / want);
-        int nt = 0;
-        for (; cap < 128; cap += 2) {
-          nt = mxk::mpnn_pack_tiles_cap(t->atom_off.data(), t->edge_off.data(), t->n_mol, cap, h5);
-          if (nt <= want) break;
-        }
-        n_tiles = cap < 128 ? nt : mxk::mpnn_pack_tiles(t->atom_off.data(), t->edge_off.data(), t->n_mol, h5);
-      }
-    }
-    CU_TRY(drv().cuMemcpyHtoDAsync(s.tile_off, h5, (size_t)(n_tiles + 1) * 4, st));
+    memcpy(s.h_in, t->blob.data(), t->blob.size());
+    CU_TRY(drv().cuMemcpyHtoDAsync(s.in_blob, s.h_in, t->blob.size(), st));
+    const int n_tiles = t->n_tiles;
     const mx_mpnn_cfg& m = d.mpnn;
     const uint16_t* wb = reinterpret_cast<const uint16_t*>(fi->weights);
     mxk::MpnnParams k{};
@@ -815,22 +870,19 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.c1 = wb + fi->m_off[8];
     k.w2 = wb + fi->m_off[9];
     k.c2 = wb + fi->m_off[10];
-    k.atom_off = reinterpret_cast<const int*>(s.atom_off);
-    k.atom_type = reinterpret_cast<const uint8_t*>(s.atom_type);
-    k.edge_off = reinterpret_cast<const int*>(s.edge_off);
-    k.edges = reinterpret_cast<const uint32_t*>(s.edges);
+    k.atom_off = reinterpret_cast<const int*>(s.in_blob + t->off_ao);
+    k.atom_type = reinterpret_cast<const uint8_t*>(s.in_blob + t->off_at);
+    k.edge_off = reinterpret_cast<const int*>(s.in_blob + t->off_eo);
+    k.edges = reinterpret_cast<const uint32_t*>(s.in_blob + t->off_ed);
     k.out = reinterpret_cast<float*>(s.d_out);
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
     k.h_stamps = reinterpret_cast<unsigned long long*>(s.d_stamps);
     k.done_tag = t->id;
+    k.inject_err = inject;
     k.n_ctas = e->n_ctas;
-    k.tile_off = reinterpret_cast<const int*>(s.tile_off);
+    k.tile_off = reinterpret_cast<const int*>(s.in_blob + t->off_tile);
     k.n_tiles = n_tiles;
     if (t->kind == MX_FN_MPNN_TRAIN) {
-      float* ht = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(h5) +
-                                           align_up((size_t)(t->n_mol + 1) * 4, 64));
-      memcpy(ht, t->targets.data(), (size_t)t->n_mol * 4);
-      CU_TRY(drv().cuMemcpyHtoDAsync(s.targets, ht, (size_t)t->n_mol * 4, st));
       mxk::MpnnTrainParams q{};
       q.T = m.steps;
       q.n_bonds = m.n_bond_types;
@@ -847,13 +899,14 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
       q.edge_off = k.edge_off;
       q.edges = k.edges;
       q.tile_off = k.tile_off;
-      q.targets = reinterpret_cast<const float*>(s.targets);
+      q.targets = reinterpret_cast<const float*>(s.in_blob + t->off_tg);
       q.y = reinterpret_cast<float*>(s.y);
       q.out = reinterpret_cast<float*>(s.d_out);
       q.lr = t->lr;
       q.stamps = k.stamps;
       q.h_stamps = k.h_stamps;
       q.done_tag = t->id;
+      q.inject_err = inject;
       if (mxk::launch_mpnn_train(q, st)) {
         set_error("mpnn training launch failed");
         return MX_EDEVICE;
@@ -1224,11 +1277,7 @@ mx_status mx_shutdown(void) {
     CtxGuard cg(L->gpus[p->gpu]->primary);
     if (p->cur) drv().cuStreamSynchronize(p->cur->stream);
     for (auto& kv : p->insts)
-      for (Slot& s : kv.second->slots) {
-        if (s.h_in) drv().cuMemFreeHost(s.h_in);
-        if (s.h_out) drv().cuMemFreeHost(s.h_out);
-        if (s.h_stamps) drv().cuMemFreeHost(s.h_stamps);
-      }
+      for (Slot& s : kv.second->slots) free_slot_host(s);
     for (auto& e : p->draining) destroy_exec(e.get());
     destroy_exec(p->cur.get());
     p->arena.release();
@@ -1394,6 +1443,7 @@ mx_status part_resize(int32_t part, int32_t sm_count, uint64_t hbm_bytes) {
   }
   Partition& p = *L->parts[part];
   Gpu& g = *L->gpus[p.gpu];
+  std::lock_guard<std::mutex> llk(p.load_mu);   // a cold start keeps p.cur until it ends
   std::vector<int> groups;
   int smc = 0;
   bool whole = false;
@@ -1459,6 +1509,7 @@ mx_status part_destroy(int32_t part) {
   }
   Partition& p = *L->parts[part];
   Gpu& g = *L->gpus[p.gpu];
+  std::lock_guard<std::mutex> llk(p.load_mu);   // no cold start in progress
   {
     std::lock_guard<std::mutex> glk(g.mu);
     if (!p.fifo.empty() || !p.inflight.empty() || !p.draining.empty()) {
@@ -1469,12 +1520,10 @@ mx_status part_destroy(int32_t part) {
   }
   CtxGuard cg(g.primary);
   drv().cuStreamSynchronize(p.cur->stream);
-  for (auto& kv : p.insts)
-    for (Slot& s : kv.second->slots) {
-      if (s.h_in) drv().cuMemFreeHost(s.h_in);
-      if (s.h_out) drv().cuMemFreeHost(s.h_out);
-      if (s.h_stamps) drv().cuMemFreeHost(s.h_stamps);
-    }
+  for (auto& kv : p.insts) {
+    for (Slot& s : kv.second->slots) free_slot_host(s);
+    if (kv.second->shared_weights) release_shared_ref(g, kv.first);
+  }
   p.insts.clear();
   release_exec(g, std::move(p.cur));
   p.arena.release();
@@ -1591,19 +1640,27 @@ mx_status fn_submit(int32_t part, const mx_task_desc* task, uint64_t* out_task) 
     t->out_tokens = task->out_tokens;
     t->out_logits = task->out_logits;
   } else {
+    // copy the inputs once, straight into their device image (caller may free on return)
+    const bool train = t->kind == MX_FN_MPNN_TRAIN;
     t->n_mol = task->n_mol;
     t->n_atoms = task->n_atoms;
     t->n_edges = task->n_edges;
-    t->atom_off.assign(task->atom_off, task->atom_off + t->n_mol + 1);
-    t->edge_off.assign(task->edge_off, task->edge_off + t->n_mol + 1);
-    t->atom_type.assign(task->atom_type, task->atom_type + t->n_atoms);
-    const uint8_t* eb = reinterpret_cast<const uint8_t*>(task->edges);
-    t->edges.assign(eb, eb + (size_t)t->n_edges * 6);
+    t->blob.resize(mpnn_blob_layout(*t, train, t->n_mol, t->n_atoms, t->n_edges));
+    uint8_t* b = t->blob.data();
+    memcpy(b + t->off_ao, task->atom_off, (size_t)(t->n_mol + 1) * 4);
+    memcpy(b + t->off_eo, task->edge_off, (size_t)(t->n_mol + 1) * 4);
+    memcpy(b + t->off_at, task->atom_type, (size_t)t->n_atoms);
+    if (t->n_edges > 0) memcpy(b + t->off_ed, task->edges, (size_t)t->n_edges * 6);
     t->out_ip = task->out_ip;
-    if (t->kind == MX_FN_MPNN_TRAIN) {
-      t->targets.assign(task->targets, task->targets + t->n_mol);
+    if (train) {
+      memcpy(b + t->off_tg, task->targets, (size_t)t->n_mol * 4);
       t->lr = task->lr;
       t->out_loss = task->out_loss;
+      // training tiles are full 128-atom tiles, independent of the partition
+      // (per-tile gradient partials are summed in tile order)
+      t->n_tiles = mxk::mpnn_pack_tiles(task->atom_off, task->edge_off, t->n_mol,
+                                        reinterpret_cast<int*>(b + t->off_tile));
+      t->tile_ctas = -2;
     }
   }
   Task* raw = t.get();
@@ -1628,6 +1685,15 @@ mx_status fn_submit(int32_t part, const mx_task_desc* task, uint64_t* out_task) 
     L->tasks[t->id] = std::move(t);
     std::lock_guard<std::mutex> glk(g->mu);
     p->fifo.push_back(raw);
+    if (raw->kind == MX_FN_MPNN) raw->tile_ctas = p->cur->n_ctas;   // balance for this size
+  }
+  if (raw->kind == MX_FN_MPNN) {
+    // inference tiling, outside every lock (the task is not `ready` yet); the
+    // dispatcher re-balances only if the partition is resized before launch
+    uint8_t* b = raw->blob.data();
+    raw->n_tiles = balanced_tiles(reinterpret_cast<const int*>(b + raw->off_ao),
+                                  reinterpret_cast<const int*>(b + raw->off_eo), raw->n_mol,
+                                  raw->tile_ctas, reinterpret_cast<int*>(b + raw->off_tile));
   }
   // cold start on first use (outside the global lock; FIFO order is kept by `ready`)
   FnInst* fi = nullptr;
@@ -1799,6 +1865,15 @@ mx_status mx_decode_profile(int32_t part, uint64_t* out, int32_t n_words) {
   CtxGuard cg(L->gpus[p->gpu]->primary);
   CU_TRY(drv().cuStreamSynchronize(p->cur->stream));
   CU_TRY(drv().cuMemcpyDtoH(out, p->sys + 65536, (size_t)n_words * 8));
+  return MX_OK;
+}
+
+mx_status mx_debug_inject_error(int32_t part, int32_t code) {
+  MX_REQUIRE_INIT();
+  if (code <= 0) return MX_EINVAL;
+  std::lock_guard<std::mutex> lk(L->mu);
+  if (!L->sched->is_live(part)) return MX_EINVAL;
+  L->parts[part]->inject_err.store(code);
   return MX_OK;
 }
 

@@ -56,13 +56,16 @@ struct Task {
   std::vector<int32_t> prompt;
   int32_t* out_tokens = nullptr;
   float* out_logits = nullptr;
-  // mpnn
+  // mpnn: the task's inputs packed at submit time in their device image (one
+  // H2D copy at launch): atom_off | edge_off | tile_off | targets (training) |
+  // atom_type | edges, each 64-byte aligned (offsets below, bytes).
   int n_mol = 0, n_atoms = 0, n_edges = 0;
-  std::vector<int32_t> atom_off, edge_off;
-  std::vector<uint8_t> atom_type, edges;
+  std::vector<uint8_t> blob;
+  uint32_t off_ao = 0, off_eo = 0, off_tile = 0, off_tg = 0, off_at = 0, off_ed = 0;
+  int n_tiles = 0;
+  int tile_ctas = -1;         // CTA count the inference tiling was balanced for
   float* out_ip = nullptr;
   // mpnn training step (N4)
-  std::vector<float> targets;
   float lr = 0.f;
   float* out_loss = nullptr;
   // execution
@@ -86,10 +89,10 @@ struct Slot {
   // decode
   CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kacc = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
               logits = 0;
-  // mpnn
-  CUdeviceptr atom_off = 0, atom_type = 0, edge_off = 0, edges = 0, out = 0, tile_off = 0;
+  // mpnn: device image of a task's packed inputs (Task::blob)
+  CUdeviceptr in_blob = 0;
   // mpnn training (N4)
-  CUdeviceptr targets = 0, y = 0, partials = 0, hsave = 0;
+  CUdeviceptr y = 0, partials = 0, hsave = 0;
   // common
   CUdeviceptr bar = 0, stamps = 0, err = 0;
   uint64_t bar_count = 0;
@@ -148,6 +151,7 @@ struct Partition {
   std::map<int, std::unique_ptr<FnInst>> insts;
   std::mutex load_mu;
   uint64_t launches = 0;
+  std::atomic<int> inject_err{0};   // mx_debug_inject_error: next launched task reports it
 };
 
 struct Gpu {

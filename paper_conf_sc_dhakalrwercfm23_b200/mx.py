@@ -103,6 +103,7 @@ _SIGS = {
     "mx_probe_smids_concurrent": (C.c_int32, [C.POINTER(C.c_int32), C.c_int32, C.c_int32,
                                               C.c_uint64, C.POINTER(C.c_uint32)]),
     "mx_launch_count": (C.c_int32, [C.POINTER(C.c_uint64)]),
+    "mx_debug_inject_error": (C.c_int32, [C.c_int32, C.c_int32]),
     "mx_decode_profile": (C.c_int32, [C.c_int32, C.POINTER(C.c_uint64), C.c_int32]),
     "mx_sched_new": (C.c_void_p, [C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_uint64]),
     "mx_sched_free": (None, [C.c_void_p]),
@@ -381,6 +382,11 @@ def decode_profile(part: int, n_ctas: int) -> np.ndarray:
     _check(lib().mx_decode_profile(part, out.ctypes.data_as(C.POINTER(C.c_uint64)), n_ctas * 8),
            "mx_decode_profile")
     return out.reshape(n_ctas, 8)
+
+
+def debug_inject_error(part: int, code: int = 7):
+    """Fault-path test hook: the next task launched on `part` reports device error `code`."""
+    _check(lib().mx_debug_inject_error(part, code), "mx_debug_inject_error")
 
 
 def launch_count() -> int:

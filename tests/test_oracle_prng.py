@@ -43,6 +43,28 @@ def test_weight_values_bf16_exact_and_uniform_levels():
     assert chi2 < 400, chi2       # 255 dof: mean 255, sd ~22.6
 
 
+def test_chunked_levels_equal_the_scalar_definition():
+    """The chunked, threaded generator (1 Mi-element chunks) equals the scalar
+    definition w_i = ((draw(key(seed, tid), i) >> 56) - 128) * 2^-12 at the first
+    elements, around every chunk boundary of a multi-chunk tensor, with an
+    offset, and for gains ((>> 60) - 8) * 2^-6 + 1."""
+    seed, tid = 0x7B00, 16 * 3 + 6
+    n = 3 * (1 << 20) + 77
+    w = prng.weight_values(seed, tid, n)
+    k = prng.key(seed, tid)
+    idx = [0, 1, 2, (1 << 20) - 1, 1 << 20, (1 << 20) + 1, 2 * (1 << 20), n - 1]
+    for i in idx:
+        assert w[i] == np.float32(((prng.draw_int(k, i) >> 56) - 128) * 2.0 ** -12), i
+    wo = prng.weight_values(seed, tid, 100, offset=(1 << 20) - 50)
+    assert np.array_equal(wo, w[(1 << 20) - 50:(1 << 20) + 50])
+    lv = prng.weight_levels(seed, tid, 1000)
+    assert lv.dtype == np.int8 and np.array_equal(lv.astype(np.float32) * np.float32(2.0 ** -12), w[:1000])
+    g = prng.gain_values(seed, 7, 300)
+    kg = prng.key(seed, 7)
+    for i in (0, 150, 299):
+        assert g[i] == np.float32(1 + ((prng.draw_int(kg, i) >> 60) - 8) * 2.0 ** -6)
+
+
 def test_gain_values_range_bf16_exact():
     g = prng.gain_values(0x7111, 23, 4096)
     assert is_bf16_exact(g)
@@ -112,3 +134,18 @@ def test_shuffle_is_permutation_and_fisher_yates_definition():
     k = prng.key(42, 0)
     want = ["b", "a"] if prng.draw_int(k, 0) % 2 == 0 else ["a", "b"]
     assert shuffle(["a", "b"]) == want
+
+
+def test_lazy_decode_layers_equal_eager_weights():
+    """decode_weights_lazy (int8-level cache, used for the 32-layer 7B parity
+    test) yields exactly the tensors of decode_weights."""
+    from workloads.weights import decode_weights, decode_weights_lazy
+    from workloads.configs import RAGGED
+    a, b = decode_weights(RAGGED), decode_weights_lazy(RAGGED)
+    assert len(b["layers"]) == RAGGED.n_layers
+    for la, lb in zip(a["layers"], b["layers"]):
+        assert la.keys() == lb.keys()
+        for k in la:
+            assert np.array_equal(la[k], lb[k]), k
+    for k in ("embed", "g_final", "lm_head"):
+        assert np.array_equal(a[k], b[k])

@@ -12,7 +12,7 @@ import numpy as np
 from .configs import (DecodeCfg, MpnnCfg, T_EMBED, T_WQ, T_WK, T_WV, T_WO, T_WGATE, T_WUP,
                       T_WDOWN, T_GATTN, T_GMLP, layer_tid, gfinal_tid, lmhead_tid,
                       M_EATOM, M_WB0, M_U, M_C, M_W1, M_C1, M_W2, M_C2)
-from .prng import weight_values, gain_values
+from .prng import weight_values, weight_levels, gain_values
 
 
 def matrix(seed: int, tid: int, rows: int, cols: int) -> np.ndarray:
@@ -40,6 +40,55 @@ def decode_weights(cfg: DecodeCfg) -> dict:
     return dict(
         embed=matrix(cfg.seed, T_EMBED, cfg.vocab, cfg.d_model),
         layers=[decode_layer(cfg, l) for l in range(cfg.n_layers)],
+        g_final=gain_values(cfg.seed, gfinal_tid(cfg), cfg.d_model),
+        lm_head=matrix(cfg.seed, lmhead_tid(cfg), cfg.vocab, cfg.d_model),
+    )
+
+
+class LazyDecodeLayers:
+    """The per-layer dicts of `decode_layer`, generated on first access and held
+    as int8 levels (1 byte per weight; values = level * 2^-12, exact), so a
+    32-layer 7B-shaped model (6.5 G weights) fits a test host. Indexing and
+    iteration return the same float32 arrays `decode_layer` would."""
+
+    _MATS = (("wq", T_WQ, "q", "d"), ("wk", T_WK, "kv", "d"), ("wv", T_WV, "kv", "d"),
+             ("wo", T_WO, "d", "q"), ("w_gate", T_WGATE, "ff", "d"), ("w_up", T_WUP, "ff", "d"),
+             ("w_down", T_WDOWN, "d", "ff"))
+
+    def __init__(self, cfg: DecodeCfg):
+        self.cfg = cfg
+        self._lv = {}
+
+    def __len__(self):
+        return self.cfg.n_layers
+
+    def _dims(self):
+        c = self.cfg
+        return {"q": c.q_dim, "kv": c.kv_dim, "d": c.d_model, "ff": c.d_ff}
+
+    def __getitem__(self, l: int) -> dict:
+        if not 0 <= l < self.cfg.n_layers:
+            raise IndexError(l)
+        c, dims = self.cfg, self._dims()
+        if l not in self._lv:
+            self._lv[l] = {name: weight_levels(c.seed, layer_tid(l, t), dims[r] * dims[k])
+                           for name, t, r, k in self._MATS}
+        out = {name: (self._lv[l][name].astype(np.float32) * np.float32(2.0 ** -12)).reshape(
+            dims[r], dims[k]) for name, t, r, k in self._MATS}
+        out["g_attn"] = gain_values(c.seed, layer_tid(l, T_GATTN), c.d_model)
+        out["g_mlp"] = gain_values(c.seed, layer_tid(l, T_GMLP), c.d_model)
+        return out
+
+    def __iter__(self):
+        for l in range(len(self)):
+            yield self[l]
+
+
+def decode_weights_lazy(cfg: DecodeCfg) -> dict:
+    """`decode_weights` with the layers generated on demand (LazyDecodeLayers)."""
+    return dict(
+        embed=matrix(cfg.seed, T_EMBED, cfg.vocab, cfg.d_model),
+        layers=LazyDecodeLayers(cfg),
         g_final=gain_values(cfg.seed, gfinal_tid(cfg), cfg.d_model),
         lm_head=matrix(cfg.seed, lmhead_tid(cfg), cfg.vocab, cfg.d_model),
     )
