@@ -68,10 +68,10 @@ def task_bytes(cfg, B, P, G):
 class ClockSampler:
     """nvidia-smi clocks + throttle reasons sampled during the timed region."""
 
-    def __init__(self, gpu: int):
-        self.gpu = gpu
+    def __init__(self, gpus):
+        self.gpus = [gpus] if isinstance(gpus, int) else list(gpus)
         self.proc = None
-        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_gpu{gpu}.csv")
+        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_gpu{self.gpus[0]}.csv")
 
     def __enter__(self):
         os.makedirs(os.path.dirname(self.path), exist_ok=True)
@@ -80,7 +80,8 @@ class ClockSampler:
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
         try:
             self.f = open(self.path, "w")
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={q}",
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", ",".join(map(str, self.gpus)),
+                                          f"--query-gpu={q}",
                                           "--format=csv,noheader,nounits", "-lms", "200"],
                                          stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
@@ -113,7 +114,7 @@ class ClockSampler:
         if not sm:
             return None
         return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx_, "reasons": sorted(reasons),
-                "samples": len(sm)}
+                "samples": len(sm), "gpus": self.gpus}
 
 
 # ---------------------------------------------------------------------------
@@ -131,17 +132,37 @@ def max_over_ranks(values, dist):
     return [float(v) for v in t]
 
 
-def make_layout(mx, gpu, n, kind):
+def sum_over_ranks(values, dist):
+    """Element-wise sum of per-rank counts (tasks, GPUs) over ranks."""
+    if not dist:
+        return [float(v) for v in values]
+    import torch
+    t = torch.tensor([float(v) for v in values], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return [float(v) for v in t]
+
+
+def local_devices(n_gpus: int, world: int, local_rank: int):
+    """Device ordinals this process drives: one per rank under torchrun
+    (world > 1), else all N requested GPUs in this process (one dispatcher
+    thread per GPU, global placement over every partition of every GPU)."""
+    if world > 1:
+        return [local_rank]
+    return list(range(max(1, n_gpus)))
+
+
+def make_layout(mx, gpus, n, kind):
+    """The same partition layout on every library GPU; partitions ordered by
+    (gpu, part id) as the STATIC rule orders them."""
     sizes = (LAYOUTS_FILL if kind == "fill" else LAYOUTS_EQUAL)[n]
-    parts = [mx.part_create(gpu, s, QUOTA) for s in sizes]
-    return parts
+    return [mx.part_create(g, s, QUOTA) for g in gpus for s in sizes]
 
 
 def run_batch(mx, fn, parts, n_tasks, equal_sizes, prompts):
     """Submit a closed batch (all at t0) and wait for all. Returns per-task results."""
     tasks = []
     for k in range(1, n_tasks + 1):
-        t = mx.decode_task(fn, prompts[k - 1], G_LEN)
+        t = mx.decode_task(fn, prompts[(k - 1) % len(prompts)], G_LEN)
         part = parts[(k - 1) % len(parts)] if equal_sizes else mx.MX_PART_ANY
         mx.fn_submit(part, t)
         tasks.append(t)
@@ -158,87 +179,87 @@ def summarize(res, n_steps):
     t_end = max(r["t_end_ns"] for r in res)
     comp = [(r["t_end_ns"] - r["t_submit_ns"]) / 1e6 for r in res]
     serv = [(r["t_end_ns"] - r["t_start_ns"]) / 1e6 for r in res]
+    per_gpu = {}
+    for r in res:
+        g = per_gpu.setdefault(r["gpu"], [r["t_start_ns"], r["t_end_ns"], 0])
+        g[0], g[1], g[2] = min(g[0], r["t_start_ns"]), max(g[1], r["t_end_ns"]), g[2] + 1
     return dict(span_s=(t_end - t_start) / 1e9, wall_s=(t_end - t_sub0) / 1e9,
                 p50_ms=float(np.percentile(comp, 50)), p99_ms=float(np.percentile(comp, 99)),
                 service_p50_ms=float(np.percentile(serv, 50)),
                 service_p99_ms=float(np.percentile(serv, 99)),
-                kernel_ms_mean=float(np.mean([r["kernel_ns"] for r in res]) / 1e6))
+                kernel_ms_mean=float(np.mean([r["kernel_ns"] for r in res]) / 1e6),
+                per_gpu={g: dict(span_s=(v[1] - v[0]) / 1e9, tasks=v[2])
+                         for g, v in sorted(per_gpu.items())})
+
+
+def choose_layout(args, sweep):
+    if args.layout == "auto":
+        return max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 37
+    return int(args.layout)
 
 
 def gpu_arm(args, rank, world, local_rank, dist):
     from paper_conf_sc_dhakalrwercfm23_b200 import mx
-    mx.mx_init([local_rank])
-    gpu = 0
+    devices = local_devices(args.gpus, world, local_rank)
+    mx.mx_init(devices)
+    gpus = list(range(len(devices)))          # library GPU indices
+    ng = len(gpus)
     cfg = GPT2S
     fn = mx.fn_register(mx.decode_desc(cfg))
     prompts = [prompt_tokens(k, 1, P_LEN, cfg.vocab) for k in range(1, N_TASKS + 1)]
     bytes_task = task_bytes(cfg, 1, P_LEN, G_LEN)
     peak, peak_src = peaks()
+    n_step = N_TASKS * ng                     # tasks per step in this process
 
     def load(parts):
         for p in parts:
             mx.fn_load(fn, p)
 
+    def sweep_one(n, kind):
+        parts = make_layout(mx, gpus, n, kind)
+        load(parts)
+        sizes = (LAYOUTS_FILL if kind == "fill" else LAYOUTS_EQUAL)[n]
+        eq = len(set(sizes)) == 1
+        tasks = sweep_tasks * ng
+        run_batch(mx, fn, parts, min(tasks, 2 * len(parts)), eq, prompts)   # warm
+        res, _ = run_batch(mx, fn, parts, tasks, eq, prompts)
+        s = summarize(res, 1)
+        for p in parts:
+            mx.part_destroy(p)
+        return dict(partitions=n, sms=sizes, tasks=tasks, tasks_per_s=tasks / s["span_s"],
+                    p50_ms=s["p50_ms"], p99_ms=s["p99_ms"],
+                    hbm_frac=tasks * bytes_task / s["span_s"] / (peak * 1e9 * ng))
+
     # --- partition sweep (Fig. 4 analog: 1 vs 2/4/7/14 partitions) ----------------
-    sweep = []
     sweep_tasks = 148
-    for n in (args.sweep if args.sweep else []):
-        parts = make_layout(mx, gpu, n, "fill")
-        load(parts)
-        eq = len(set(LAYOUTS_FILL[n])) == 1
-        run_batch(mx, fn, parts, min(sweep_tasks, 2 * len(parts)), eq, prompts)   # warm
-        res, _ = run_batch(mx, fn, parts, sweep_tasks, eq, prompts)
-        s = summarize(res, 1)
-        sweep.append(dict(partitions=n, sms=LAYOUTS_FILL[n], tasks=sweep_tasks,
-                          tasks_per_s=sweep_tasks / s["span_s"], p50_ms=s["p50_ms"],
-                          p99_ms=s["p99_ms"],
-                          hbm_frac=sweep_tasks * bytes_task / s["span_s"] / (peak * 1e9)))
-        for p in parts:
-            mx.part_destroy(p)
+    sweep = [sweep_one(n, "fill") for n in args.sweep]
     # equal (MIG-like) layouts of the same N: STATIC (k-1) mod N placement
-    sweep_equal = []
-    for n in (args.sweep if args.sweep else []):
-        if n not in LAYOUTS_EQUAL or n == 1:
-            continue
-        parts = make_layout(mx, gpu, n, "equal")
-        load(parts)
-        run_batch(mx, fn, parts, min(sweep_tasks, 2 * len(parts)), True, prompts)   # warm
-        res, _ = run_batch(mx, fn, parts, sweep_tasks, True, prompts)
-        s = summarize(res, 1)
-        sweep_equal.append(dict(partitions=n, sms=LAYOUTS_EQUAL[n], tasks=sweep_tasks,
-                                tasks_per_s=sweep_tasks / s["span_s"], p50_ms=s["p50_ms"],
-                                p99_ms=s["p99_ms"],
-                                hbm_frac=sweep_tasks * bytes_task / s["span_s"] / (peak * 1e9)))
-        for p in parts:
-            mx.part_destroy(p)
-    if args.layout == "auto":
-        n_main = max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 14
-    else:
-        n_main = int(args.layout)
+    sweep_equal = [sweep_one(n, "equal") for n in args.sweep if n in LAYOUTS_EQUAL and n != 1]
+    n_main = choose_layout(args, sweep)
 
     # --- main timed run ------------------------------------------------------------
-    parts = make_layout(mx, gpu, n_main, "fill")
+    parts = make_layout(mx, gpus, n_main, "fill")
     load(parts)
     eq = len(set(LAYOUTS_FILL[n_main])) == 1
     for _ in range(args.warmup):
-        run_batch(mx, fn, parts, N_TASKS, eq, prompts)
+        run_batch(mx, fn, parts, n_step, eq, prompts)
     if dist:
         dist.barrier()
     l0 = mx.launch_count()
     all_res = []
-    with ClockSampler(local_rank) as clk:
+    with ClockSampler(devices) as clk:
         h0 = time.perf_counter()
         for _ in range(args.steps):
-            res, _ = run_batch(mx, fn, parts, N_TASKS, eq, prompts)
+            res, _ = run_batch(mx, fn, parts, n_step, eq, prompts)
             all_res += res
         h1 = time.perf_counter()
     launches = mx.launch_count() - l0
     if dist:
         dist.barrier()
     s = summarize(all_res, args.steps)
-    span = s["span_s"]
-    wall = h1 - h0
-    span, wall = max_over_ranks([span, wall], dist)
+    span, wall = max_over_ranks([s["span_s"], h1 - h0], dist)
+    n_total, gpus_total, launches_total = sum_over_ranks([n_step * args.steps, ng, launches], dist)
+    n_total, gpus_total = int(n_total), int(gpus_total)
     priv_held = sum(mx.part_query(p)["hbm_used"] for p in parts)
     for p in parts:
         mx.part_destroy(p)
@@ -246,22 +267,22 @@ def gpu_arm(args, rank, world, local_rank, dist):
     n3 = None
     if args.n3:
         fs = mx.fn_register(mx.decode_desc(cfg, shared_weights=True))
-        sparts = [mx.part_create(gpu, sz, 64 << 20) for sz in LAYOUTS_FILL[n_main]]
+        sparts = [mx.part_create(g, sz, 64 << 20) for g in gpus for sz in LAYOUTS_FILL[n_main]]
         for p in sparts:
             mx.fn_load(fs, p)
         held = sum(mx.part_query(p)["hbm_used"] for p in sparts) + \
-            mx.weight_pool_query(gpu)["used_bytes"]
-        run_batch(mx, fs, sparts, N_TASKS, eq, prompts)   # warm
+            sum(mx.weight_pool_query(g)["used_bytes"] for g in gpus)
+        run_batch(mx, fs, sparts, n_step, eq, prompts)   # warm
         n3_steps = min(args.steps, 2)
         n3_res = []
         for _ in range(n3_steps):
-            r, _ = run_batch(mx, fs, sparts, N_TASKS, eq, prompts)
+            r, _ = run_batch(mx, fs, sparts, n_step, eq, prompts)
             n3_res += r
         s3 = summarize(n3_res, n3_steps)
         (span3,) = max_over_ranks([s3["span_s"]], dist)
-        v3 = N_TASKS * n3_steps * world / span3
+        v3 = n_total / args.steps * n3_steps / span3
         n3 = {"tasks_per_s": round(v3, 3), "steps": n3_steps,
-              "hbm_frac_algorithmic": round(bytes_task * v3 / world / 1e9 / peak, 4),
+              "hbm_frac_algorithmic": round(bytes_task * v3 / gpus_total / 1e9 / peak, 4),
               "p50_ms": round(s3["p50_ms"], 3), "p99_ms": round(s3["p99_ms"], 3),
               "hbm_held_gib": round(held / 2**30, 3),
               "private_hbm_held_gib": round(priv_held / 2**30, 3),
@@ -274,50 +295,50 @@ def gpu_arm(args, rank, world, local_rank, dist):
     mx.mx_shutdown()
     if rank != 0:
         return None
-    n_total = N_TASKS * args.steps * world
     value = n_total / span
-    agg_bytes = bytes_task * N_TASKS * args.steps * world
-    achieved_gbs = agg_bytes / span / 1e9 / world   # per GPU
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "decode_traffic.json")
-    if os.path.exists(tp):
-        try:
-            traffic = json.load(open(tp)).get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    achieved_gbs = bytes_task * n_total / span / 1e9 / gpus_total   # per GPU
     out = {
-        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": gpus_total,
         "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(span / args.steps * 1e3, 3), "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "bf16 weights/KV, fp32 math",
         "data": "synthetic (seeded bf16 weights generated on device, seeded prompts)",
         "config": {"workload": "configs[1]: GPT-2-small-shaped Llama decode, batch 1, P=16, G=32",
                    "model": "gpt2s-llama (L12 d768 H12 d_ff2048 V50257)",
-                   "tasks_per_step_per_gpu": N_TASKS, "partitions": n_main,
+                   "tasks_per_step_per_gpu": N_TASKS, "partitions_per_gpu": n_main,
                    "partition_sms": LAYOUTS_FILL[n_main],
-                   "placement": "STATIC (k-1) mod P" if eq else "WLAW (C5)",
-                   "parallelism": f"replicas x{world} (independent tasks, no collective)",
+                   "placement": ("STATIC (k-1) mod P" if eq else "WLAW (C5)") +
+                                (" over all partitions of all GPUs" if ng > 1 else ""),
+                   "parallelism": (f"replicas x{gpus_total}: " +
+                                   (f"{world} ranks (torchrun), one GPU each" if world > 1 else
+                                    f"one process, {ng} GPU dispatcher threads") +
+                                   " (independent tasks, no collective)"),
                    "l2": "inputs larger than L2: 324 MB of weights per partition copy"},
         "p50_ms": round(s["p50_ms"], 3), "p99_ms": round(s["p99_ms"], 3),
         "service_p50_ms": round(s["service_p50_ms"], 3),
         "service_p99_ms": round(s["service_p99_ms"], 3),
         "gen_tok_per_s": round(value * G_LEN, 1),
         "hbm_frac": round(achieved_gbs / peak, 4),
+        "per_gpu": [{"gpu": devices[g], "tasks": v["tasks"], "span_s": round(v["span_s"], 4),
+                     "hbm_frac": round(v["tasks"] * bytes_task / v["span_s"] / 1e9 / peak, 4)}
+                    for g, v in s["per_gpu"].items()],
         "partitions_sweep": sweep,
         "partitions_sweep_equal": sweep_equal,
         "roofline": {"bound": "hbm", "achieved": round(achieved_gbs, 1), "peak": peak,
-                     "unit": "GB/s", "frac": round(achieved_gbs / peak, 4), "traffic": traffic,
+                     "unit": "GB/s", "frac": round(achieved_gbs / peak, 4),
+                     "traffic": decode_traffic(),
                      "kernel": "decode_kernel (persistent megakernel, all partitions together)",
                      "algorithmic_bytes_per_launch": bytes_task,
                      "kernel_ms_mean_per_launch": round(s["kernel_ms_mean"], 3),
                      "peak_source": peak_src},
         "e2e": {"value": round(n_total / wall, 3), "unit": UNIT,
-                "h2d_bytes_per_step": N_TASKS * world * P_LEN * 4,
-                "d2h_bytes_per_step": N_TASKS * world * (G_LEN * 4 + 24)},
-        "gpu_launches": int(launches) * world,
-        "timing": "value: device %globaltimer span (first kernel start -> last kernel end) "
-                  "over the K steps, max over ranks; kernel_ms from CUDA events on each "
-                  "partition's stream; e2e: host wall clock fn_submit -> last fn_wait",
+                "h2d_bytes_per_step": int(n_total / args.steps) * P_LEN * 4,
+                "d2h_bytes_per_step": int(n_total / args.steps) * (G_LEN * 4 + 24)},
+        "gpu_launches": int(launches_total),
+        "timing": "value: device %globaltimer span (first kernel start -> last kernel end, "
+                  "over all GPUs of the process) over the K steps, max over ranks; kernel_ms "
+                  "from the kernels' own timestamps; e2e: host wall clock fn_submit -> last "
+                  "fn_wait (prompts H2D, tokens D2H inside)",
     }
     if sweep:
         base = [d for d in sweep if d["partitions"] == 1]
@@ -327,9 +348,31 @@ def gpu_arm(args, rank, world, local_rank, dist):
     if n3:
         out["n3_shared_weights"] = n3
     out["clocks"] = clk.summary()
-    if args.cpu_baseline and world == 1:
+    if args.cpu_baseline and gpus_total == 1:
         out["cpu_baseline"] = cpu_baseline(args)
     return out
+
+
+def decode_traffic():
+    """dram bytes per decode launch from the committed ncu capture, only if it
+    was taken on the current kernel source (stamp = hash of decode_impl.cuh)."""
+    tp = os.path.join(ROOT, "profiles", "decode_traffic.json")
+    try:
+        d = json.load(open(tp))
+    except Exception:
+        return None
+    if d.get("source_sha256") != kernel_source_hash():
+        return None
+    return d.get("dram_bytes_per_launch")
+
+
+def kernel_source_hash():
+    import hashlib
+    h = hashlib.sha256()
+    for f in ("decode_impl.cuh", "common.cuh"):
+        with open(os.path.join(ROOT, "paper_conf_sc_dhakalrwercfm23_b200", "csrc", "kernels", f), "rb") as fh:
+            h.update(fh.read())
+    return h.hexdigest()
 
 
 # ---------------------------------------------------------------------------
