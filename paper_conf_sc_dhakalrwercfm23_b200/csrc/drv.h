@@ -56,6 +56,7 @@ namespace mx {
   X(cuLaunchKernel)                \
   X(cuLaunchCooperativeKernel)     \
   X(cuKernelSetAttribute)          \
+  X(cuTensorMapEncodeTiled)        \
   X(cuGetErrorString)
 
 struct Drv {

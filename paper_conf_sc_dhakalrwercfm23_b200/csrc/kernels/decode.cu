@@ -14,9 +14,11 @@ template <int B>
 int set_attrs_b(int device);
 
 int decode_smem_bytes(int B, int kmax, int* n_stages) {
-  const int fixed = decode_xin_bytes(B, kmax) + kConsumerWarps * 3 * kAttHd * 4 + 8 * 8 +
-                    8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 128;
-  const int per_stage = kStageBytes + decode_red_floats(B) * 4 + kMaxUnits * 4 + 16;
+  // 1024-byte alignment slack + activation operand + attention scratch +
+  // mbarriers (TMEM slots) + small scratch; the rest is the weight ring
+  const int fixed = 1024 + decode_act_bytes(B, kmax) + kConsumerWarps * 3 * kAttHd * 4 +
+                    4 * 2 * 8 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 16;
+  const int per_stage = kBoxBytes + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;
   if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;
@@ -25,8 +27,6 @@ int decode_smem_bytes(int B, int kmax, int* n_stages) {
   return ns * per_stage + fixed;
 }
 
-// Fused (per-CTA) attention only for small attention on the CUDA-core path
-// (the tensor-core path stages its activations as bf16 hi/lo, not fp32).
 int decode_prof_buckets() {
 #ifdef MX_PROF_BUCKETS
   return 1;
@@ -42,7 +42,7 @@ int decode_prof_buckets() {
 // grid barrier per layer but replicates the K/V reads over the grid: used for
 // small attention on grids of at most MX_FUSE_MAX_CTAS CTAs.
 int decode_fuse_attention(int B, int H, int hd, int n_ctas) {
-  return (B < kTcMinBatch && B * H * hd <= 1024 && n_ctas <= MX_FUSE_MAX_CTAS) ? 1 : 0;
+  return (B * H * hd <= 1024 && n_ctas <= MX_FUSE_MAX_CTAS) ? 1 : 0;
 }
 
 uint64_t decode_barriers(int L, int P, int G, int fuse_att) {

@@ -6,55 +6,51 @@
 
 namespace mxk {
 
-#ifndef MX_STAGE_KB
-#define MX_STAGE_KB 32
-#endif
 #ifndef MX_CONSUMER_WARPS
 #define MX_CONSUMER_WARPS 11
 #endif
 #ifndef MX_MAX_STAGES
-#define MX_MAX_STAGES 6
+#define MX_MAX_STAGES 12
 #endif
-#ifndef MX_ROWS_B1
-#define MX_ROWS_B1 4
-#endif
-constexpr int kStageBytes = MX_STAGE_KB * 1024;   // one TMA bulk stage of weight rows
-constexpr int kConsumerWarps = MX_CONSUMER_WARPS;   // GEMV / attention warps per CTA
+// Decode GEMVs run on the 5th-generation tensor cores (tcgen05): D[rows][16] =
+// W[rows][K] . X[16][K]^T with W (bf16 weights, the A operand, M = 128 rows
+// per MMA) streamed by 3-D tiled TMA in K-major SWIZZLE_128B boxes of
+// [128 rows][64 columns] (16 KiB = one ring stage) and X (the activations as
+// a bf16 hi/lo pair per sequence, the B operand) staged in shared memory.
+constexpr int kTileM = 128;             // weight rows per MMA tile (UMMA M)
+constexpr int kBlkK = 64;               // K columns per TMA box (128 bytes)
+constexpr int kBoxBytes = kTileM * kBlkK * 2;   // one ring stage
+constexpr int kConsumerWarps = MX_CONSUMER_WARPS;   // staging / attention / MMA / epilogue warps
 constexpr int kDecodeThreads = 32 * (kConsumerWarps + 1);  // + 1 producer (TMA) warp
 constexpr int kAttHd = 128;             // max attention head_dim
-constexpr int kMaxUnits = 128;          // (row, 256-col chunk) work units per tile
 constexpr int kMaxCtas = 160;           // >= 148 SMs
 constexpr int kMaxSeqCap = 512;         // attention keeps <= 16 scores per lane
-constexpr int kXinSegBytes = 64 * 1024; // activation staging per K segment (B * cols * 4)
-// Columns of one K segment for batch B: phases whose B*K*4 exceeds the staging
-// capacity run as several K segments (split-K inside the owning CTA).
+// Tensor maps of one decode function instance (device global memory, 64-byte
+// aligned CUtensorMap objects): 6 matrices (QKV, O, GATE, UP, DOWN, LM) x 3 box
+// heights (128, 32, 8 rows; a CTA's row range is decomposed into them).
+constexpr int kDecodeMats = 6;
+constexpr int kDecodeBoxH = 3;
+constexpr int kDecodeMaps = kDecodeMats * kDecodeBoxH;
 #ifdef __CUDACC__
 #define MX_HD __host__ __device__
 #else
 #define MX_HD
 #endif
-MX_HD constexpr int decode_seg_cols(int B) { return (kXinSegBytes / (B * 4)) & ~255; }
-// Batch sizes >= kTcMinBatch run the GEMVs on the tensor cores (K7): tiles of
-// 8 weight rows x <= kTcCols columns (one 32 KiB stage with a 16-byte row pad).
-#ifndef MX_TC_MIN_BATCH
-#define MX_TC_MIN_BATCH 4
-#endif
-constexpr int kTcMinBatch = MX_TC_MIN_BATCH;
-#ifndef MX_TC_SPLIT
-#define MX_TC_SPLIT 3
-#endif
-// A tensor-core tile (one stage) is consumed by kTcSplit warps that split its
-// K iterations.
-constexpr int kTcSplit = MX_TC_SPLIT;
-// floats of per-stage partial-sum space (CUDA-core units: [kMaxUnits][B];
-// tensor-core tiles: the split warps' fragments, [kTcSplit][32 lanes][2])
-MX_HD constexpr int decode_red_floats(int B) {
-  return (B >= kTcMinBatch && kMaxUnits * B < kTcSplit * 64) ? kTcSplit * 64 : kMaxUnits * B;
-}
-constexpr int kTcCols = 2016;
-// Activation staging columns for the widest phase input kmax.
-MX_HD constexpr int decode_xin_cols(int B, int kmax) {
-  return ((kmax + 255) & ~255) < decode_seg_cols(B) ? ((kmax + 255) & ~255) : decode_seg_cols(B);
+// Activation operand: B <= 4 -> one 8-row swizzle atom per 64 columns (hi of
+// sequence b in row b, lo in row 4 + b; the N = 16 MMA reads the atom twice,
+// stride byte offset 0); B > 4 -> two atoms (hi rows 0-7, lo rows 8-15).
+MX_HD constexpr int decode_act_rows(int B) { return B <= 4 ? 8 : 16; }
+MX_HD constexpr int decode_act_lo(int B) { return B <= 4 ? 4 : 8; }
+MX_HD constexpr int decode_act_blk_bytes(int B) { return decode_act_rows(B) * 128; }
+// Columns of one K segment: phases whose input is wider than 64 KiB of operand
+// run as several K segments (split-K inside the owning CTA).
+MX_HD constexpr int decode_seg_cols(int B) { return (64 * 1024 / decode_act_blk_bytes(B)) * kBlkK; }
+MX_HD constexpr int decode_act_bytes(int B, int kmax) {
+  return ((((kmax + kBlkK - 1) / kBlkK) * kBlkK < decode_seg_cols(B)
+               ? ((kmax + kBlkK - 1) / kBlkK) * kBlkK
+               : decode_seg_cols(B)) /
+          kBlkK) *
+         decode_act_blk_bytes(B);
 }
 
 // One decode task on one partition: all P+G-1 steps in ONE persistent launch
@@ -90,7 +86,8 @@ struct DecodeParams {
   unsigned long long bar_base;
   unsigned long long* stamps;  // [2] globaltimer start / end
   int* err;                  // 0 ok, 1 barrier timeout
-  unsigned long long* prof;  // [n_ctas][8] cycle buckets (MX_DECODE_PROF=1) or nullptr
+  unsigned long long* prof;  // [n_ctas][16] cycle buckets (MX_DECODE_PROF=1) or nullptr
+  const void* tmaps;         // kDecodeMaps CUtensorMap (device memory): [matrix][box height]
   // host-mapped completion record: [0] start, [1] end, [2] err, [3] = done_tag,
   // written last (after a system-scope fence) by CTA 0
   unsigned long long* h_stamps;
@@ -105,15 +102,8 @@ int decode_prof_buckets();
 // Number of grid barriers one decode launch performs (host bookkeeping of bar_base).
 uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 
-// Shared-memory bytes of the decode kernel for a given shape.
+// Shared-memory bytes of the decode kernel for a given shape (-1: does not fit).
 int decode_smem_bytes(int B, int kmax, int* n_stages);
-// Bytes of the activation staging buffer (CUDA-core: fp32 [B][cols]; tensor
-// cores: bf16 hi and lo [B][cols + 8] plus a 64-byte zero block).
-MX_HD constexpr int decode_xin_bytes(int B, int kmax) {
-  return B >= kTcMinBatch
-             ? 2 * B * ((((kmax + 31) & ~31) < kTcCols ? ((kmax + 31) & ~31) : kTcCols) * 2 + 16) + 64
-             : B * decode_xin_cols(B, kmax) * 4;
-}
 
 // cooperative != 0: cuLaunchCooperativeKernel (all CTAs co-resident; used on
 // unpartitioned streams where other kernels compete for the same SMs).

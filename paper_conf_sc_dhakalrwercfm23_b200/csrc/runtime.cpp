@@ -164,7 +164,7 @@ static int validate_fn(const mx_fn_desc& d) {
       return MX_EINVAL;
     }
     if (c.d_model > 8192 || c.d_ff > 16384 || q > 16384) {
-      set_error("decode cfg: a weight row must fit one 32 KiB TMA stage");
+      set_error("decode cfg: d_model <= 8192, q_dim and d_ff <= 16384");
       return MX_EINVAL;
     }
     const int kmax = std::max(std::max(c.d_model, q), c.d_ff);
@@ -607,6 +607,45 @@ static void release_shared_ref(Gpu& gpu, int fn_id) {
   gpu.shared_w.clear();
 }
 
+// 3-D tiled TMA descriptors of a decode instance's weights (kernels.h
+// kDecodeMaps): per matrix kind (QKV, O, GATE, UP, DOWN, LM) a tensor of
+// {K columns, R rows, L layers} bf16 (layer stride = the layer block), boxes
+// of 64 columns x {128, 32, 8} rows, K-major SWIZZLE_128B (the UMMA A-operand
+// layout); out-of-bounds rows / columns are zero-filled.
+static int encode_decode_maps(const FnInst& fi, std::vector<CUtensorMap>& maps) {
+  const mx_decode_cfg& c = fi.fn->desc.dec;
+  const uint64_t d = c.d_model, q = (uint64_t)c.n_heads * c.head_dim,
+                 kv = (uint64_t)c.n_kv_heads * c.head_dim, ff = c.d_ff, V = c.vocab;
+  struct Mat {
+    uint64_t off, K, R;
+    bool layered;
+  } mats[mxk::kDecodeMats] = {{fi.off_wqkv, d, q + 2 * kv, true}, {fi.off_wo, q, d, true},
+                              {fi.off_wgate, d, ff, true},         {fi.off_wup, d, ff, true},
+                              {fi.off_wdown, ff, d, true},         {fi.off_lm, d, V, false}};
+  static const cuuint32_t box_rows[mxk::kDecodeBoxH] = {128, 32, 8};
+  maps.resize(mxk::kDecodeMaps);
+  uint16_t* w = reinterpret_cast<uint16_t*>(fi.weights);
+  for (int m = 0; m < mxk::kDecodeMats; ++m) {
+    const Mat& M = mats[m];
+    const cuuint64_t dims[3] = {M.K, M.R, M.layered ? (cuuint64_t)c.n_layers : 1};
+    const cuuint64_t strides[2] = {M.K * 2, M.layered ? fi.layer_stride * 2 : M.K * M.R * 2};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    for (int h = 0; h < mxk::kDecodeBoxH; ++h) {
+      const cuuint32_t box[3] = {(cuuint32_t)mxk::kBlkK, box_rows[h], 1};
+      CUresult r = drv().cuTensorMapEncodeTiled(
+          &maps[m * mxk::kDecodeBoxH + h], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, w + M.off, dims,
+          strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      if (r != CUDA_SUCCESS) {
+        set_error("cuTensorMapEncodeTiled (matrix %d, box %u rows) failed: %s", m, box_rows[h],
+                  cu_str(r));
+        return MX_EDEVICE;
+      }
+    }
+  }
+  return MX_OK;
+}
+
 // Caller holds p.load_mu (part_resize / part_destroy take it too, so p.cur and
 // its stream stay fixed while the load runs). Synchronous cold start on the
 // partition's stream.
@@ -688,6 +727,16 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
     if (rc) return fail(rc);
   }
   if (!fi->shared_weights && (rc = generate_weights(*fi, st, nct))) return fail(rc);
+  std::vector<CUtensorMap> maps;
+  if (d.kind == MX_FN_DECODE) {
+    if ((rc = encode_decode_maps(*fi, maps))) return fail(rc);
+    const uint64_t mb = maps.size() * sizeof(CUtensorMap);
+    if ((rc = alloc_ptr(p, mb, &fi->tmaps))) return fail(rc);
+    if (drv().cuMemcpyHtoDAsync(fi->tmaps, maps.data(), mb, st) != CUDA_SUCCESS) {
+      set_error("tensor map upload failed");
+      return fail(MX_EDEVICE);
+    }
+  }
   if (d.kind == MX_FN_MPNN_TRAIN) {
     // fp32 training state, widened exactly from the seeded bf16 values (N4)
     if (mxk::launch_widen_bf16(reinterpret_cast<float*>(fi->params),
@@ -829,6 +878,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.stamps = reinterpret_cast<unsigned long long*>(s.stamps);
     k.err = reinterpret_cast<int*>(s.err);
     k.prof = g_decode_prof ? reinterpret_cast<unsigned long long*>(p.sys + 65536) : nullptr;
+    k.tmaps = reinterpret_cast<const void*>(fi->tmaps);
     if (!t->use_flag) CU_TRY(drv().cuEventRecord(ev[0], st));
     int rc = mxk::launch_decode(k, st, e->shared ? 1 : 0);
     if (rc) {

@@ -119,6 +119,7 @@ struct FnInst {
   CUdeviceptr weights = 0;
   uint64_t weight_bytes = 0;
   CUdeviceptr rope = 0;
+  CUdeviceptr tmaps = 0;         // decode: mxk::kDecodeMaps CUtensorMap over the weights
   // decode layout (elements)
   uint64_t layer_stride = 0, off_wqkv = 0, off_wo = 0, off_wgate = 0, off_wup = 0, off_wdown = 0,
            off_gattn = 0, off_gmlp = 0, off_gfinal = 0, off_lm = 0, off_embed = 0;

@@ -50,12 +50,11 @@ for k in range(a.tasks):
 if os.environ.get("MX_DECODE_PROF") == "1":
     n = mx.part_query(p)["n_ctas"]
     pr = mx.decode_profile(p, 2 * n).astype(float).reshape(n, 16)
-    names = ["total", "grid_barrier", "stage_input", "ring_wait(c0)", "gemv", "attention",
-             "producer_wait", "-"]
+    names = {0: "total", 1: "grid_barrier", 2: "stage_input", 3: "mma_wait_full", 4: "gemv(mma+epi)",
+             5: "attention", 6: "producer_wait", 7: "mma_wait_acc", 8: "epi_wait_tfull"}
     tot = pr[:, 0].mean()
-    print(f"  unit latency (warp0) {pr[:, 7].sum() / max(pr[:, 8].sum(), 1):.0f} cyc over {pr[:, 8].mean():.0f} units/CTA")
-    for i, nm in enumerate(names[:7]):
-        print(f"  {nm:14s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
+    for i, nm in names.items():
+        print(f"  {nm:16s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
               f"  min {pr[:, i].min() / 1e6:8.2f} max {pr[:, i].max() / 1e6:8.2f}")
 mx.part_destroy(p)
 mx.mx_shutdown()
