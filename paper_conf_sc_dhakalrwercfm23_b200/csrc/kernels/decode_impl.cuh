@@ -52,6 +52,9 @@ constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
 constexpr int kMmaWarp = 1;                 // warp whose lane 0 issues the MMAs
 constexpr int kEpiWarp0 = 2;                // warps 2..5 drain TMEM (lane quarter = warp % 4)
 constexpr int kAccSlots = 4;                // TMEM accumulator slots of 32 columns
+#ifndef MX_MMA_WARP
+#define MX_MMA_WARP 1                       // 1: warp-uniform issue, elected lane (see tc05.cuh)
+#endif
 constexpr uint32_t kTmemCols = 32 * kAccSlots;
 static_assert(kConsumerWarps >= 5, "MMA warp + 4 epilogue warps");
 
@@ -351,11 +354,10 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
                                           long long& w_full, long long& w_acc) {
   constexpr uint32_t idesc = umma_idesc_bf16(kTileM, 16);
   constexpr uint32_t sbo = (B <= 4) ? 0u : 1024u;   // B <= 4: the 8-row atom is read twice
-  const uint64_t act_desc = umma_desc_sw128(smem_u32(sm.act), sbo);
-  const uint64_t ring_desc = umma_desc_sw128(smem_u32(sm.ring));
-  constexpr uint64_t kActBlk = (uint64_t)(decode_act_blk_bytes(B) >> 4);   // descriptor units
-  constexpr uint64_t kBoxUnits = (uint64_t)(kBoxBytes >> 4);
+  const uint32_t act0 = smem_u32(sm.act), ring0 = smem_u32(sm.ring);
   const int nm = (ph.kind == PH_GU) ? 2 : 1;
+  const bool lane0 = (threadIdx.x & 31) == 0;
+  (void)lane0;
   int r0, r1;
   my_rows(ph.R, p.n_ctas, blockIdx.x, k, &r0, &r1);
   for (int rt = r0; rt < r1; rt += kTileM) {
@@ -367,27 +369,42 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
     tc_fence_after();
     const uint32_t dcol = tmem_base + slot * 32u;
     for (int kb = 0; kb < ph.nkb; ++kb) {
-      const uint64_t bd = act_desc + (uint64_t)kb * kActBlk;
+      const uint64_t bd = umma_desc_sw128(act0 + (uint32_t)(kb * decode_act_blk_bytes(B)), sbo);
       for (int m = 0; m < nm; ++m) {
         const long long tf = MX_CLK();
         mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
         __syncwarp();
         w_full += MX_CLK() - tf;
         tc_fence_after();
-        const uint64_t ad = ring_desc + (uint64_t)stage * kBoxUnits;
+        const uint64_t ad = umma_desc_sw128(ring0 + stage * (uint32_t)kBoxBytes);
         const uint32_t d = dcol + 16u * (uint32_t)m;
+#if MX_MMA_WARP
 #pragma unroll
         for (int j = 0; j < kBlkK / 16; ++j)
           umma_f16_warp(d, ad + 2u * (uint32_t)j, bd + 2u * (uint32_t)j, idesc,
                         (kb > 0 || j > 0) ? 1u : 0u);
         umma_commit_warp(smem_u32(&sm.empty[stage]));   // stage free once these MMAs completed
+#else
+        if (lane0) {
+#pragma unroll
+          for (int j = 0; j < kBlkK / 16; ++j)
+            umma_f16(d, ad + 2u * (uint32_t)j, bd + 2u * (uint32_t)j, idesc, (kb > 0 || j > 0) ? 1u : 0u);
+          umma_commit(smem_u32(&sm.empty[stage]));
+        }
+        __syncwarp();
+#endif
         if (++stage == (uint32_t)n_stages) {
           stage = 0;
           phase_bit ^= 1u;
         }
       }
     }
+#if MX_MMA_WARP
     umma_commit_warp(smem_u32(&sm.tfull[slot]));         // accumulator ready for the epilogue
+#else
+    if (lane0) umma_commit(smem_u32(&sm.tfull[slot]));
+    __syncwarp();
+#endif
     ++tc;
   }
 }
@@ -413,6 +430,7 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
     ++tc;
     const long long tw = MX_CLK();
     mbar_wait_bounded(&sm.tfull[slot], use & 1u, p.err);
+    __syncwarp();   // tcgen05.ld is .sync.aligned: the warp must be converged
     w_tf += MX_CLK() - tw;
     tc_fence_after();
     const uint32_t taddr = tmem_base + ((uint32_t)(32 * q) << 16) + slot * 32u;
