@@ -65,11 +65,14 @@ static_assert(kConsumerWarps >= 5, "MMA warp + 4 epilogue warps");
 #endif
 // Bounded mbarrier wait: a launch that would otherwise hang (a protocol error
 // or a failed copy) raises *err after 4 s and stops waiting, so the task
-// completes with MX_EDEVICE instead of wedging its partition.
+// completes with MX_EDEVICE instead of wedging its partition. SPIN = 1 polls
+// without the suspend hint (lower wake-up latency for the pipeline roles).
+template <int SPIN = 0>
 __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity, int* err) {
-  if (MX_FULL_WAIT(bar, parity)) return;
+  auto done = [&]() { return SPIN ? mbar_try_wait(bar, parity) : MX_FULL_WAIT(bar, parity); };
+  if (done()) return;
   const uint64_t t0 = globaltimer();
-  while (!MX_FULL_WAIT(bar, parity)) {
+  while (!done()) {
     if (ld_volatile_i32(err)) return;
     if (globaltimer() - t0 > 4000000000ull) {
       atomicExch(err, 1);
@@ -77,6 +80,15 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
     }
   }
 }
+#ifndef MX_WAIT_PROD
+#define MX_WAIT_PROD 1
+#endif
+#ifndef MX_WAIT_MMA
+#define MX_WAIT_MMA 1
+#endif
+#ifndef MX_WAIT_EPI
+#define MX_WAIT_EPI 0
+#endif
 
 // Per-CTA cycle buckets (MX_DECODE_PROF=1) exist only in profiling builds
 // (MX_DEFS=-DMX_PROF_BUCKETS).
@@ -311,7 +323,7 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
             const int col = ph.k0 + kb * kBlkK;
             for (int m = 0; m < nm; ++m) {
               const long long tw = MX_CLK();
-              mbar_wait_bounded(&sm.empty[stage], phase_bit ^ 1u, p.err);
+              mbar_wait_bounded<MX_WAIT_PROD>(&sm.empty[stage], phase_bit ^ 1u, p.err);
               wait_cyc += MX_CLK() - tw;
               // the box bytes (OOB rows / columns arrive zero-filled and count)
               mbar_arrive_expect_tx(&sm.full[stage], (uint32_t)h8 * 128u);
@@ -363,7 +375,7 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
   for (int rt = r0; rt < r1; rt += kTileM) {
     const uint32_t slot = tc % kAccSlots, use = tc / kAccSlots;
     const long long ta = MX_CLK();
-    mbar_wait_bounded(&sm.tempty[slot], (use & 1u) ^ 1u, p.err);
+    mbar_wait_bounded<MX_WAIT_MMA>(&sm.tempty[slot], (use & 1u) ^ 1u, p.err);
     __syncwarp();
     w_acc += MX_CLK() - ta;
     tc_fence_after();
@@ -372,7 +384,7 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
       const uint64_t bd = umma_desc_sw128(act0 + (uint32_t)(kb * decode_act_blk_bytes(B)), sbo);
       for (int m = 0; m < nm; ++m) {
         const long long tf = MX_CLK();
-        mbar_wait_bounded(&sm.full[stage], phase_bit, p.err);
+        mbar_wait_bounded<MX_WAIT_MMA>(&sm.full[stage], phase_bit, p.err);
         __syncwarp();
         w_full += MX_CLK() - tf;
         tc_fence_after();
@@ -429,7 +441,7 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
     const uint32_t slot = tc % kAccSlots, use = tc / kAccSlots;
     ++tc;
     const long long tw = MX_CLK();
-    mbar_wait_bounded(&sm.tfull[slot], use & 1u, p.err);
+    mbar_wait_bounded<MX_WAIT_EPI>(&sm.tfull[slot], use & 1u, p.err);
     __syncwarp();   // tcgen05.ld is .sync.aligned: the warp must be converged
     w_tf += MX_CLK() - tw;
     tc_fence_after();
