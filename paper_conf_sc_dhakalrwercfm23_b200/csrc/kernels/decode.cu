@@ -18,7 +18,7 @@ int decode_smem_bytes(int B, int kmax, int* n_stages) {
   // mbarriers (TMEM slots) + small scratch; the rest is the weight ring
   const int fixed = 1024 + decode_act_bytes(B, kmax) + kConsumerWarps * 3 * kAttHd * 4 +
                     4 * 2 * 8 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 16;
-  const int per_stage = kBoxBytes + 16;
+  const int per_stage = kStageBytes + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;
   if (ns > MX_MAX_STAGES) ns = MX_MAX_STAGES;

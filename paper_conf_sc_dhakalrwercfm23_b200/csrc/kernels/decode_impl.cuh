@@ -122,7 +122,8 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
   }
   constexpr int SEG = decode_seg_cols(B);
   ph.nseg = max(1, (ph.KF + SEG - 1) / SEG);
-  const int w = round64((ph.KF + ph.nseg - 1) / ph.nseg);
+  const int w = (ph.nseg == 1) ? round64(ph.KF)
+                               : ((ph.KF + ph.nseg - 1) / ph.nseg + kSegGrain - 1) / kSegGrain * kSegGrain;
   ph.seg = seg;
   ph.k0 = seg * w;
   ph.K = min(w, ph.KF - ph.k0);
@@ -158,7 +159,7 @@ __device__ __forceinline__ int phase_kind(int k, int L, int fuse_att) {
 }
 
 struct Smem {
-  uint8_t* ring;             // [n_stages][kBoxBytes] weight boxes (1024-aligned)
+  uint8_t* ring;             // [n_stages][kStageBytes] weight boxes (1024-aligned)
   uint8_t* act;              // activation operand (B rows hi + B rows lo, SWIZZLE_128B)
   float* att;                // [kConsumerWarps][3][kAttHd]
   uint64_t* full;            // [n_stages] TMA -> MMA
@@ -177,7 +178,7 @@ __device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax) {
   Smem s;
   uint8_t* p = raw + ((1024 - (smem_u32(raw) & 1023)) & 1023);
   s.ring = p;
-  p += (size_t)n_stages * kBoxBytes;
+  p += (size_t)n_stages * kStageBytes;
   s.act = p;
   p += (size_t)decode_act_bytes(B, kmax);
   s.att = reinterpret_cast<float*>(p);
@@ -265,8 +266,9 @@ __device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned lon
   named_bar_sync(1, kNCT);
 }
 
-__device__ __forceinline__ const void* tmap(const DecodeParams& p, int mat, int hsel) {
-  return reinterpret_cast<const uint8_t*>(p.tmaps) + (size_t)(mat * kDecodeBoxH + hsel) * 128;
+// tensor map of matrix `mat` with box height h8 (a multiple of 8, <= 128)
+__device__ __forceinline__ const void* tmap(const DecodeParams& p, int mat, int h8) {
+  return reinterpret_cast<const uint8_t*>(p.tmaps) + (size_t)(mat * kDecodeBoxH + (h8 >> 3) - 1) * 128;
 }
 
 // ---------------------------------------------------------------------------
@@ -282,7 +284,8 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
   uint32_t stage = 0, phase_bit = 0;
   long long wait_cyc = 0;
   const uint64_t pol = policy_evict_first();
-  for (int i = 0; i < kDecodeMaps; ++i) prefetch_tensormap(tmap(p, i / kDecodeBoxH, i % kDecodeBoxH));
+  for (int i = 0; i < kDecodeMaps; ++i)
+    prefetch_tensormap(reinterpret_cast<const uint8_t*>(p.tmaps) + (size_t)i * 128);
   const uint32_t ring0 = smem_u32(sm.ring);
   for (int s = 0; s < S; ++s) {
     const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
@@ -319,27 +322,17 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
         my_rows(ph.R, C, cta, k, &r0, &r1);
         for (int rt = r0; rt < r1; rt += kTileM) {
           const int h8 = (min(kTileM, r1 - rt) + 7) & ~7;
-          for (int kb = 0; kb < ph.nkb; ++kb) {
-            const int col = ph.k0 + kb * kBlkK;
+          const int nk = decode_box_blocks(h8);
+          const uint32_t bytes = (uint32_t)(h8 * nk * 128);
+          for (int kb = 0; kb < ph.nkb; kb += nk) {
             for (int m = 0; m < nm; ++m) {
               const long long tw = MX_CLK();
               mbar_wait_bounded<MX_WAIT_PROD>(&sm.empty[stage], phase_bit ^ 1u, p.err);
               wait_cyc += MX_CLK() - tw;
-              // the box bytes (OOB rows / columns arrive zero-filled and count)
-              mbar_arrive_expect_tx(&sm.full[stage], (uint32_t)h8 * 128u);
-              const uint32_t dst = ring0 + stage * (uint32_t)kBoxBytes;
-              const int mat = ph.mat + m;
-              if (h8 == kTileM) {
-                tma_load_3d(dst, tmap(p, mat, 0), col, rt, ph.lz, &sm.full[stage], pol);
-              } else {
-                int o = 0;
-                for (; o + 32 <= h8; o += 32)
-                  tma_load_3d(dst + (uint32_t)o * 128u, tmap(p, mat, 1), col, rt + o, ph.lz,
-                              &sm.full[stage], pol);
-                for (; o < h8; o += 8)
-                  tma_load_3d(dst + (uint32_t)o * 128u, tmap(p, mat, 2), col, rt + o, ph.lz,
-                              &sm.full[stage], pol);
-              }
+              // the full box (blocks past K are out of bounds: zero-filled, counted)
+              mbar_arrive_expect_tx(&sm.full[stage], bytes);
+              tma_load_4d(ring0 + stage * (uint32_t)kStageBytes, tmap(p, ph.mat + m, h8), 0, rt,
+                          ph.k0 / kBlkK + kb, ph.lz, &sm.full[stage], pol);
               if (++stage == (uint32_t)n_stages) {
                 stage = 0;
                 phase_bit ^= 1u;
@@ -380,29 +373,43 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
     w_acc += MX_CLK() - ta;
     tc_fence_after();
     const uint32_t dcol = tmem_base + slot * 32u;
-    for (int kb = 0; kb < ph.nkb; ++kb) {
-      const uint64_t bd = umma_desc_sw128(act0 + (uint32_t)(kb * decode_act_blk_bytes(B)), sbo);
+    const int h8 = (min(kTileM, r1 - rt) + 7) & ~7;
+    const int nk = decode_box_blocks(h8);
+    for (int kb = 0; kb < ph.nkb; kb += nk) {
+      const int nkc = min(nk, ph.nkb - kb);
       for (int m = 0; m < nm; ++m) {
         const long long tf = MX_CLK();
         mbar_wait_bounded<MX_WAIT_MMA>(&sm.full[stage], phase_bit, p.err);
         __syncwarp();
         w_full += MX_CLK() - tf;
         tc_fence_after();
-        const uint64_t ad = umma_desc_sw128(ring0 + stage * (uint32_t)kBoxBytes);
         const uint32_t d = dcol + 16u * (uint32_t)m;
+        const uint32_t sa = ring0 + stage * (uint32_t)kStageBytes;
+        for (int j = 0; j < nkc; ++j) {
+          // block j of the box: [h8 rows][128 B]; an M = 128 MMA on a tail tile
+          // also reads the rows after it (garbage rows -> discarded outputs)
+          const uint64_t ad = umma_desc_sw128(sa + (uint32_t)(j * h8 * 128));
+          const uint64_t bd =
+              umma_desc_sw128(act0 + (uint32_t)((kb + j) * decode_act_blk_bytes(B)), sbo);
 #if MX_MMA_WARP
 #pragma unroll
-        for (int j = 0; j < kBlkK / 16; ++j)
-          umma_f16_warp(d, ad + 2u * (uint32_t)j, bd + 2u * (uint32_t)j, idesc,
-                        (kb > 0 || j > 0) ? 1u : 0u);
+          for (int jj = 0; jj < kBlkK / 16; ++jj)
+            umma_f16_warp(d, ad + 2u * (uint32_t)jj, bd + 2u * (uint32_t)jj, idesc,
+                          (kb + j > 0 || jj > 0) ? 1u : 0u);
+#else
+          if (lane0) {
+#pragma unroll
+            for (int jj = 0; jj < kBlkK / 16; ++jj)
+              umma_f16(d, ad + 2u * (uint32_t)jj, bd + 2u * (uint32_t)jj, idesc,
+                       (kb + j > 0 || jj > 0) ? 1u : 0u);
+          }
+          __syncwarp();
+#endif
+        }
+#if MX_MMA_WARP
         umma_commit_warp(smem_u32(&sm.empty[stage]));   // stage free once these MMAs completed
 #else
-        if (lane0) {
-#pragma unroll
-          for (int j = 0; j < kBlkK / 16; ++j)
-            umma_f16(d, ad + 2u * (uint32_t)j, bd + 2u * (uint32_t)j, idesc, (kb > 0 || j > 0) ? 1u : 0u);
-          umma_commit(smem_u32(&sm.empty[stage]));
-        }
+        if (lane0) umma_commit(smem_u32(&sm.empty[stage]));
         __syncwarp();
 #endif
         if (++stage == (uint32_t)n_stages) {

@@ -6,6 +6,12 @@
 
 namespace mxk {
 
+#ifdef __CUDACC__
+#define MX_HD __host__ __device__
+#else
+#define MX_HD
+#endif
+#define MX_HD_FWD MX_HD
 #ifndef MX_CONSUMER_WARPS
 #define MX_CONSUMER_WARPS 11
 #endif
@@ -18,24 +24,26 @@ namespace mxk {
 // [128 rows][64 columns] (16 KiB = one ring stage) and X (the activations as
 // a bf16 hi/lo pair per sequence, the B operand) staged in shared memory.
 constexpr int kTileM = 128;             // weight rows per MMA tile (UMMA M)
-constexpr int kBlkK = 64;               // K columns per TMA box (128 bytes)
-constexpr int kBoxBytes = kTileM * kBlkK * 2;   // one ring stage
+constexpr int kBlkK = 64;               // K columns per swizzle-atom row (128 bytes)
+constexpr int kStageBytes = 32 * 1024;  // one ring stage: a tile's rows x up to 8 column blocks
+// Column blocks per TMA box for a tile of h8 rows (h8 a multiple of 8): the
+// box is [blocks][h8 rows][64 columns], so each row's nk*128 contiguous bytes
+// are fetched by one request.
+// (a power of two <= 8 dividing the 512-column segment grain).
+MX_HD_FWD constexpr int decode_box_blocks(int h8) {
+  return h8 <= 32 ? 8 : h8 <= 64 ? 4 : h8 <= 128 ? 2 : 1;
+}
 constexpr int kConsumerWarps = MX_CONSUMER_WARPS;   // staging / attention / MMA / epilogue warps
 constexpr int kDecodeThreads = 32 * (kConsumerWarps + 1);  // + 1 producer (TMA) warp
 constexpr int kAttHd = 128;             // max attention head_dim
 constexpr int kMaxCtas = 160;           // >= 148 SMs
 constexpr int kMaxSeqCap = 512;         // attention keeps <= 16 scores per lane
 // Tensor maps of one decode function instance (device global memory, 64-byte
-// aligned CUtensorMap objects): 6 matrices (QKV, O, GATE, UP, DOWN, LM) x 3 box
-// heights (128, 32, 8 rows; a CTA's row range is decomposed into them).
+// aligned CUtensorMap objects): 6 matrices (QKV, O, GATE, UP, DOWN, LM) x 16
+// box heights (8..128 rows): 4-D {64 columns, rows, column blocks, layers}.
 constexpr int kDecodeMats = 6;
-constexpr int kDecodeBoxH = 3;
+constexpr int kDecodeBoxH = 16;
 constexpr int kDecodeMaps = kDecodeMats * kDecodeBoxH;
-#ifdef __CUDACC__
-#define MX_HD __host__ __device__
-#else
-#define MX_HD
-#endif
 // Activation operand: B <= 4 -> one 8-row swizzle atom per 64 columns (hi of
 // sequence b in row b, lo in row 4 + b; the N = 16 MMA reads the atom twice,
 // stride byte offset 0); B > 4 -> two atoms (hi rows 0-7, lo rows 8-15).
@@ -45,6 +53,7 @@ MX_HD constexpr int decode_act_blk_bytes(int B) { return decode_act_rows(B) * 12
 // Columns of one K segment: phases whose input is wider than 64 KiB of operand
 // run as several K segments (split-K inside the owning CTA).
 MX_HD constexpr int decode_seg_cols(int B) { return (64 * 1024 / decode_act_blk_bytes(B)) * kBlkK; }
+constexpr int kSegGrain = 8 * kBlkK;   // K segment widths are multiples of 512 columns
 MX_HD constexpr int decode_act_bytes(int B, int kmax) {
   return ((((kmax + kBlkK - 1) / kBlkK) * kBlkK < decode_seg_cols(B)
                ? ((kmax + kBlkK - 1) / kBlkK) * kBlkK

@@ -566,6 +566,11 @@ static int generate_weights(FnInst& fi, CUstream st, int nct) {
     for (int k = 0; k <= 10; ++k)
       if (!(k >= 1 && k <= 4 && k - 1 >= d.mpnn.n_bond_types)) tids.push_back(k);
   }
+  // alignment padding between tensors reads as 0 (decode TMA boxes may touch it)
+  if (drv().cuMemsetD8Async(fi.weights, 0, fi.weight_bytes, st) != CUDA_SUCCESS) {
+    set_error("weight block clear failed");
+    return MX_EDEVICE;
+  }
   for (int tid : tids) {
     uint64_t off, n;
     int gain;
@@ -607,11 +612,16 @@ static void release_shared_ref(Gpu& gpu, int fn_id) {
   gpu.shared_w.clear();
 }
 
-// 3-D tiled TMA descriptors of a decode instance's weights (kernels.h
-// kDecodeMaps): per matrix kind (QKV, O, GATE, UP, DOWN, LM) a tensor of
-// {K columns, R rows, L layers} bf16 (layer stride = the layer block), boxes
-// of 64 columns x {128, 32, 8} rows, K-major SWIZZLE_128B (the UMMA A-operand
-// layout); out-of-bounds rows / columns are zero-filled.
+// 4-D tiled TMA descriptors of a decode instance's weights (kernels.h
+// kDecodeMaps): per matrix kind (QKV, O, GATE, UP, DOWN, LM) and per box
+// height h = 8, 16, ..., 128 rows, the tensor {64 columns, R rows,
+// ceil(K/64) column blocks, L layers} bf16 with strides {2K, 128, layer
+// block} bytes and a box of {64, h, decode_box_blocks(h), 1}: one request
+// fetches h rows x (blocks x 128 B) contiguous bytes per row, landing as
+// [blocks][h rows][128 B] in K-major SWIZZLE_128B (the UMMA A-operand layout).
+// Rows >= R and blocks >= ceil(K/64) are zero-filled; a last block that is
+// partly past K reads the following (finite, zero-padded) weight elements,
+// which meet zero activations.
 static int encode_decode_maps(const FnInst& fi, std::vector<CUtensorMap>& maps) {
   const mx_decode_cfg& c = fi.fn->desc.dec;
   const uint64_t d = c.d_model, q = (uint64_t)c.n_heads * c.head_dim,
@@ -622,22 +632,25 @@ static int encode_decode_maps(const FnInst& fi, std::vector<CUtensorMap>& maps) 
   } mats[mxk::kDecodeMats] = {{fi.off_wqkv, d, q + 2 * kv, true}, {fi.off_wo, q, d, true},
                               {fi.off_wgate, d, ff, true},         {fi.off_wup, d, ff, true},
                               {fi.off_wdown, ff, d, true},         {fi.off_lm, d, V, false}};
-  static const cuuint32_t box_rows[mxk::kDecodeBoxH] = {128, 32, 8};
   maps.resize(mxk::kDecodeMaps);
   uint16_t* w = reinterpret_cast<uint16_t*>(fi.weights);
   for (int m = 0; m < mxk::kDecodeMats; ++m) {
     const Mat& M = mats[m];
-    const cuuint64_t dims[3] = {M.K, M.R, M.layered ? (cuuint64_t)c.n_layers : 1};
-    const cuuint64_t strides[2] = {M.K * 2, M.layered ? fi.layer_stride * 2 : M.K * M.R * 2};
-    const cuuint32_t estr[3] = {1, 1, 1};
+    const cuuint64_t dims[4] = {(cuuint64_t)mxk::kBlkK, M.R, (M.K + mxk::kBlkK - 1) / mxk::kBlkK,
+                                M.layered ? (cuuint64_t)c.n_layers : 1};
+    const cuuint64_t strides[3] = {M.K * 2, 128,
+                                   M.layered ? fi.layer_stride * 2 : align_up(M.K * M.R * 2, 256)};
+    const cuuint32_t estr[4] = {1, 1, 1, 1};
     for (int h = 0; h < mxk::kDecodeBoxH; ++h) {
-      const cuuint32_t box[3] = {(cuuint32_t)mxk::kBlkK, box_rows[h], 1};
+      const int rows = 8 * (h + 1);
+      const cuuint32_t box[4] = {(cuuint32_t)mxk::kBlkK, (cuuint32_t)rows,
+                                 (cuuint32_t)mxk::decode_box_blocks(rows), 1};
       CUresult r = drv().cuTensorMapEncodeTiled(
-          &maps[m * mxk::kDecodeBoxH + h], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, w + M.off, dims,
+          &maps[m * mxk::kDecodeBoxH + h], CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, w + M.off, dims,
           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
       if (r != CUDA_SUCCESS) {
-        set_error("cuTensorMapEncodeTiled (matrix %d, box %u rows) failed: %s", m, box_rows[h],
+        set_error("cuTensorMapEncodeTiled (matrix %d, box %d rows) failed: %s", m, rows,
                   cu_str(r));
         return MX_EDEVICE;
       }
