@@ -11,9 +11,11 @@ One bench step = one closed batch of N_TASKS tasks submitted through the C ABI
 (fn_submit with host prompt buffers) and collected with fn_wait (host token
 buffers) on the chosen partition layout of each GPU. Before the timed run a
 short sweep measures the 1 / 2 / 4 / 7 / 14-partition layouts (D0 "fill") and
-the finer 18 / 37-partition layouts (4-SM groups); the timed run uses the best.
+the finer 18 / 37-partition layouts (4-SM groups) — the paper's Fig. 4
+comparison; the timed run's layout is chosen by N2 right-sizing (fn_rightsize:
+the task measured alone on each candidate size).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--layout auto|1|2|4|7|14]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--layout auto|sweep|1|2|4|7|14|18|37]
     python bench.py --impl reference      # the CPU oracle on a bounded sample
 
 Multi-GPU (torchrun, one rank per GPU): tasks are independent, so every rank
@@ -155,7 +157,15 @@ def make_layout(mx, gpus, n, kind):
     """The same partition layout on every library GPU; partitions ordered by
     (gpu, part id) as the STATIC rule orders them."""
     sizes = (LAYOUTS_FILL if kind == "fill" else LAYOUTS_EQUAL)[n]
+    return make_sized(mx, gpus, sizes)
+
+
+def make_sized(mx, gpus, sizes):
     return [mx.part_create(g, s, QUOTA) for g in gpus for s in sizes]
+
+
+# N2 right-sizing candidates (SM counts; 4-SM group multiples, SURVEY.md §8(f) N2)
+N2_CAND = [4, 8, 12, 16, 20, 24, 36, 40, 48, 72, 148]
 
 
 def run_batch(mx, fn, parts, n_tasks, equal_sizes, prompts):
@@ -192,10 +202,23 @@ def summarize(res, n_steps):
                          for g, v in sorted(per_gpu.items())})
 
 
-def choose_layout(args, sweep):
+def choose_layout(mx, fn, args, sweep, prompts):
+    """Partition sizes of the timed run. 'auto' = N2 right-sizing (fn_rightsize:
+    the task measured alone on each candidate size, throughput objective);
+    'sweep' = the best fill layout of the D2 sweep; an integer = that fill layout."""
     if args.layout == "auto":
-        return max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 37
-    return int(args.layout)
+        sample = mx.decode_task(fn, prompts[0], G_LEN)
+        r = mx.fn_rightsize(fn, 0, sample, N2_CAND, hbm_bytes=QUOTA, reps=2, objective=1)
+        n2 = {"chosen_sms": r["sm"], "partitions": r["parts"],
+              "predicted_tasks_per_s": round(r["rate_per_s"], 2),
+              "curve_ms": [(sm, round(t / 1e6, 3)) for sm, t in r["curve"]],
+              "rule": "mx_rightsize objective 1: argmax floor(148/s)/t(s) over the measured "
+                      "single-instance service times t(s)"}
+        return [r["sm"]] * r["parts"], n2
+    if args.layout == "sweep":
+        n = max(sweep, key=lambda d: d["tasks_per_s"])["partitions"] if sweep else 37
+        return LAYOUTS_FILL[n], None
+    return LAYOUTS_FILL[int(args.layout)], None
 
 
 def gpu_arm(args, rank, world, local_rank, dist):
@@ -235,12 +258,13 @@ def gpu_arm(args, rank, world, local_rank, dist):
     sweep = [sweep_one(n, "fill") for n in args.sweep]
     # equal (MIG-like) layouts of the same N: STATIC (k-1) mod N placement
     sweep_equal = [sweep_one(n, "equal") for n in args.sweep if n in LAYOUTS_EQUAL and n != 1]
-    n_main = choose_layout(args, sweep)
+    sizes, n2 = choose_layout(mx, fn, args, sweep, prompts)
+    n_main = len(sizes)
 
     # --- main timed run ------------------------------------------------------------
-    parts = make_layout(mx, gpus, n_main, "fill")
+    parts = make_sized(mx, gpus, sizes)
     load(parts)
-    eq = len(set(LAYOUTS_FILL[n_main])) == 1
+    eq = len(set(sizes)) == 1
     for _ in range(args.warmup):
         run_batch(mx, fn, parts, n_step, eq, prompts)
     if dist:
@@ -267,7 +291,7 @@ def gpu_arm(args, rank, world, local_rank, dist):
     n3 = None
     if args.n3:
         fs = mx.fn_register(mx.decode_desc(cfg, shared_weights=True))
-        sparts = [mx.part_create(g, sz, 64 << 20) for g in gpus for sz in LAYOUTS_FILL[n_main]]
+        sparts = [mx.part_create(g, sz, 64 << 20) for g in gpus for sz in sizes]
         for p in sparts:
             mx.fn_load(fs, p)
         held = sum(mx.part_query(p)["hbm_used"] for p in sparts) + \
@@ -306,7 +330,9 @@ def gpu_arm(args, rank, world, local_rank, dist):
         "config": {"workload": "configs[1]: GPT-2-small-shaped Llama decode, batch 1, P=16, G=32",
                    "model": "gpt2s-llama (L12 d768 H12 d_ff2048 V50257)",
                    "tasks_per_step_per_gpu": N_TASKS, "partitions_per_gpu": n_main,
-                   "partition_sms": LAYOUTS_FILL[n_main],
+                   "partition_sms": sizes,
+                   "layout": ("N2 right-sizing (fn_rightsize)" if n2 else
+                              f"fill layout {n_main}" if args.layout != "sweep" else "best of sweep"),
                    "placement": ("STATIC (k-1) mod P" if eq else "WLAW (C5)") +
                                 (" over all partitions of all GPUs" if ng > 1 else ""),
                    "parallelism": (f"replicas x{gpus_total}: " +
@@ -347,6 +373,9 @@ def gpu_arm(args, rank, world, local_rank, dist):
                                                 / base[0]["tasks_per_s"], 3)
     if n3:
         out["n3_shared_weights"] = n3
+    if n2:
+        n2["measured_tasks_per_s_per_gpu"] = round(value / gpus_total, 2)
+        out["n2_rightsize"] = n2
     out["clocks"] = clk.summary()
     if args.cpu_baseline and gpus_total == 1:
         out["cpu_baseline"] = cpu_baseline(args)

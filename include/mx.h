@@ -316,6 +316,25 @@ mx_status mx_rightsize(const int32_t* sms, const double* t, int32_t n_points, in
                        int32_t max_parts, int32_t objective, double slack, int32_t* out_sm,
                        int32_t* out_parts, double* out_rate);
 
+/* Right-sizing from a measured sweep (N2: "the dispatcher sizes partitions
+ * automatically"). For each candidate SM count cand_sms[i] (ascending; a
+ * count that rounds to an already measured group count is skipped and its
+ * out_t_ns entry left untouched) a partition of that size and `hbm_bytes`
+ * is created on `gpu`, `fn` is loaded, `sample` (a task of `fn`; its output
+ * buffers receive the results) runs once to warm up and `reps` more times,
+ * and the best device service time (t_end - t_start) is kept in out_t_ns[i]
+ * (may be NULL). The partition is destroyed before the next size, so the
+ * function runs alone (the paper's Fig. 2 SM sweep). The
+ * measured curve then goes through mx_rightsize(objective, slack) over the
+ * GPU's SM count with at most 64 partitions: *out_sm per partition,
+ * *out_parts partitions, *out_rate = out_parts / t (tasks per ns). The
+ * calibration tasks are ordinary tasks (they appear in the trace). Errors
+ * of the underlying calls are returned as is; MX_EINVAL for bad arguments. */
+mx_status fn_rightsize(int32_t fn, int32_t gpu, const mx_task_desc* sample, uint64_t hbm_bytes,
+                       const int32_t* cand_sms, int32_t n_cand, int32_t reps, int32_t objective,
+                       double slack, int32_t* out_sm, int32_t* out_parts, double* out_rate,
+                       double* out_t_ns);
+
 #ifdef __cplusplus
 }
 #endif

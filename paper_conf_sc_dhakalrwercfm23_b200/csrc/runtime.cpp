@@ -2001,6 +2001,62 @@ mx_status mx_sched_trace(const mx_sched* s, void* buf, uint64_t cap, uint64_t* l
   return MX_OK;
 }
 
+// N2: measure a function's single-instance service time on partitions of the
+// candidate sizes (one warm-up + `reps` timed runs of `sample` each, alone on
+// the GPU), then apply the right-sizing rule (mx_rightsize) to the measured
+// curve. Uses only this ABI (part_create / fn_load / fn_submit / fn_wait /
+// part_destroy), so the calibration tasks are ordinary tasks of the trace.
+mx_status fn_rightsize(int32_t fn, int32_t gpu, const mx_task_desc* sample, uint64_t hbm_bytes,
+                       const int32_t* cand_sms, int32_t n_cand, int32_t reps, int32_t objective,
+                       double slack, int32_t* out_sm, int32_t* out_parts, double* out_rate,
+                       double* out_t_ns) {
+  MX_REQUIRE_INIT();
+  if (!sample || !cand_sms || n_cand < 1 || n_cand > 64 || reps < 1 || !out_sm || !out_parts ||
+      sample->fn != fn)
+    return MX_EINVAL;
+  int sm_total = 0;
+  {
+    std::lock_guard<std::mutex> lk(L->mu);
+    if (!find_fn(L, fn)) {
+      set_error("fn_rightsize: unknown fn %d", fn);
+      return MX_EINVAL;
+    }
+    if (gpu < 0 || gpu >= (int)L->gpus.size()) return MX_ENODEV;
+    sm_total = L->gpus[gpu]->sm_total;
+  }
+  std::vector<int32_t> sms;
+  std::vector<double> t;
+  for (int i = 0; i < n_cand; ++i) {
+    if (cand_sms[i] <= 0 || (i > 0 && cand_sms[i] <= cand_sms[i - 1])) return MX_EINVAL;
+    int32_t part = -1;
+    int rc = part_create(gpu, cand_sms[i], hbm_bytes, &part);
+    if (rc) return rc;
+    mx_part_info info{};
+    part_query(part, &info);
+    if (!sms.empty() && info.sm_count <= sms.back()) {   // rounds to the same group count
+      part_destroy(part);
+      continue;
+    }
+    double best = 0.0;
+    for (int r = 0; r <= reps && rc == MX_OK; ++r) {
+      uint64_t id = 0;
+      mx_result res{};
+      rc = fn_submit(part, sample, &id);
+      if (rc == MX_OK) rc = fn_wait(id, -1, &res);
+      if (rc == MX_OK && res.status != MX_OK) rc = res.status;
+      const double ns = (double)(res.t_end_ns - res.t_start_ns);
+      if (rc == MX_OK && r > 0 && (best == 0.0 || ns < best)) best = ns;   // r = 0: warm-up
+    }
+    part_destroy(part);
+    if (rc) return rc;
+    sms.push_back(info.sm_count);
+    t.push_back(best);
+    if (out_t_ns) out_t_ns[i] = best;
+  }
+  return mx_rightsize(sms.data(), t.data(), (int32_t)sms.size(), sm_total, 64, objective, slack,
+                      out_sm, out_parts, out_rate);
+}
+
 mx_status mx_rightsize(const int32_t* sms, const double* t, int32_t n_points, int32_t total_sms,
                        int32_t max_parts, int32_t objective, double slack, int32_t* out_sm,
                        int32_t* out_parts, double* out_rate) {

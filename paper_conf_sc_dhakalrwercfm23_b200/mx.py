@@ -120,6 +120,10 @@ _SIGS = {
                                  C.c_int32, C.c_int32, C.c_double, C.POINTER(C.c_int32),
                                  C.POINTER(C.c_int32), C.POINTER(C.c_double)]),
     "mx_sched_trace": (C.c_int32, [C.c_void_p, C.c_void_p, C.c_uint64, C.POINTER(C.c_uint64)]),
+    "fn_rightsize": (C.c_int32, [C.c_int32, C.c_int32, C.POINTER(TaskDescC), C.c_uint64,
+                                 C.POINTER(C.c_int32), C.c_int32, C.c_int32, C.c_int32, C.c_double,
+                                 C.POINTER(C.c_int32), C.POINTER(C.c_int32), C.POINTER(C.c_double),
+                                 C.POINTER(C.c_double)]),
 }
 
 _lib = None
@@ -404,6 +408,20 @@ def rightsize(sms, t, total_sms=148, max_parts=37, objective=1, slack=0.0):
     _check(lib().mx_rightsize(a, b, n, total_sms, max_parts, objective, slack, C.byref(o_sm),
                               C.byref(o_p), C.byref(o_r)), "mx_rightsize")
     return o_sm.value, o_p.value, o_r.value
+
+
+def fn_rightsize(fn: int, gpu: int, sample: Task, cand_sms, hbm_bytes: int = 1 << 30,
+                 reps: int = 2, objective: int = 1, slack: float = 0.0):
+    """N2: measure `sample` alone on each candidate partition size, then right-size.
+    -> dict(sm, parts, rate_per_s, curve=[(sms, t_ns)])"""
+    n = len(cand_sms)
+    a = (C.c_int32 * n)(*[int(x) for x in cand_sms])
+    tt = (C.c_double * n)(*([0.0] * n))
+    o_sm, o_p, o_r = C.c_int32(), C.c_int32(), C.c_double()
+    _check(lib().fn_rightsize(fn, gpu, C.byref(sample.desc), hbm_bytes, a, n, reps, objective, slack,
+                              C.byref(o_sm), C.byref(o_p), C.byref(o_r), tt), "fn_rightsize")
+    return {"sm": o_sm.value, "parts": o_p.value, "rate_per_s": o_r.value * 1e9,
+            "curve": [(int(cand_sms[i]), float(tt[i])) for i in range(n) if tt[i] > 0]}
 
 
 # ---------------------------------------------------------------------------
