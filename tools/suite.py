@@ -13,7 +13,8 @@ All inputs are seeded and synthetic (workloads/); weights are generated on the
 device from seeds. Times are device %globaltimer stamps (t_start/t_end of each
 task); HBM fractions use algorithmic bytes (metrics.decode_task_bytes) over the
 device span against MEASURED_PEAKS.json. Output parity of these workloads is
-covered by tests/ (-m gpu); this tool only measures.
+covered by tests/ (-m gpu; the D5 farm's checks in tests/test_gpu_farm_d5.py);
+this tool only measures.
 """
 from __future__ import annotations
 
@@ -26,6 +27,7 @@ import time
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tools"))
 
 import numpy as np  # noqa: E402
 
@@ -243,75 +245,33 @@ def cmd_c4(a, mx):
             "peak_gbs": peak_gbs(), "peak_bf16_tflops": peak_bf16_tflops(), "layouts": rows}
 
 
-LAYOUT_B = [40, 40, 16, 16, 16, 8, 8]
-
-
-def apply_layout(mx, parts, sizes):
-    """Resize partitions to `sizes` (shrinks first so growing ones find free groups)."""
-    cur = [mx.part_query(p)["sm_count"] for p in parts]
-    order = sorted(range(len(parts)), key=lambda i: sizes[i] - cur[i])
-    lat_ms = []
-    for i in order:
-        if sizes[i] != cur[i]:
-            h0 = time.perf_counter()
-            mx.part_resize(parts[i], sizes[i], 0)
-            lat_ms.append((time.perf_counter() - h0) * 1e3)
-    return lat_ms
 
 
 def cmd_c5(a, mx):
-    fd = mx.fn_register(mx.decode_desc(GPT2S))
-    fm = mx.fn_register(mx.mpnn_desc(MPNN, MOLS, MOLS * 30, MOLS * 32))
-    mol_cache = [molecules(k, MOLS) for k in range(1, a.mol_variants + 1)]
-    mfl = float(np.mean([mpnn_task_flops(m, MPNN.hidden, MPNN.steps) for m in mol_cache]))
+    """D5 task farm (tools/farm.py). The correctness checks of the same farm run
+    (trace vs the simulator, invariants I1-I5, 2 % sampled oracle parity) are
+    tests/test_gpu_farm_d5.py: only tests/ may execute oracle/."""
+    from tools.farm import Farm, FILL7, LAYOUT_B
+    farm = Farm(mx, a.mol_variants)
+    mfl = float(np.mean([mpnn_task_flops(m, MPNN.hidden, MPNN.steps) for m in farm.mol_cache]))
     out = {"suite": "D5 c5", "workload": f"configs[4]: task farm of {a.tasks} tasks, 50/50 "
            "GPT-2s decode / MPNN, shuffled (seed 42), WLAW over 7 fill partitions, layout "
            f"alternating fill-7 <-> {LAYOUT_B} via part_resize between waves of "
            f"{a.resize_every} submissions (wave w+2 is submitted after wave w completes)",
            "peak_gbs": peak_gbs()}
-    A = LAYOUTS_FILL[7]
-    for label, sizes, n_tasks in (("partitioned", A, a.tasks), ("1_partition", [148], a.base_tasks)):
-        parts = [mx.part_create(0, s, 1 << 30) for s in sizes]
-        for p in parts:
-            mx.fn_load(fd, p)
-            mx.fn_load(fm, p)
-        warm = mixed_items(mx, fd, fm, len(parts), len(parts), mol_cache)
-        closed_batch(mx, [(mx.MX_PART_ANY, t) for _, t in warm])
-        items = mixed_items(mx, fd, fm, n_tasks // 2, n_tasks - n_tasks // 2, mol_cache)
-        resize_ms = []
-        h0 = time.perf_counter()
-        use_b = False
-        # Waves of `resize_every` submissions. Before wave w >= 2 is submitted,
-        # wave w-2 is collected and the layout flips, so every resize happens
-        # while about one wave of work is queued or running (a resize between
-        # instantaneous submissions would only ever see an idle queue).
-        W = a.resize_every
-        waves = [items[i:i + W] for i in range(0, len(items), W)]
-        res_by_wave = {}
-        for w, wave in enumerate(waves):
-            if w >= 2:
-                res_by_wave[w - 2] = [mx.fn_wait(t) for _, t in waves[w - 2]]
-                if label == "partitioned":
-                    use_b = not use_b
-                    resize_ms += apply_layout(mx, parts, LAYOUT_B if use_b else A)
-            for _, t in wave:
-                mx.fn_submit(mx.MX_PART_ANY, t)
-        for w in range(len(waves)):
-            if w not in res_by_wave:
-                res_by_wave[w] = [mx.fn_wait(t) for _, t in waves[w]]
-        res = [r for w in range(len(waves)) for r in res_by_wave[w]]
-        wall = time.perf_counter() - h0
-        assert all(r["status"] == 0 for r in res)
-        st = class_stats(res, [k for k, _ in items], mfl, n_tasks // 2, n_tasks - n_tasks // 2)
+    for label, sizes, n_tasks, every in (("partitioned", FILL7, a.tasks, a.resize_every),
+                                         ("1_partition", [148], a.base_tasks, 0)):
+        r = farm.run(sizes, n_tasks, every)
+        res = r["results"]
+        assert all(x["status"] == 0 for x in res)
+        st = class_stats(res, [k for k, _, _ in r["items"]], mfl, n_tasks // 2, n_tasks - n_tasks // 2)
         st["tasks"] = n_tasks
-        st["e2e_tasks_per_s"] = round(n_tasks / wall, 3)
-        if resize_ms:
-            st["part_resize_ms"] = {"n": len(resize_ms), **{k: round(v, 3) for k, v in
-                                                            percentiles(resize_ms).items()},
-                                    "max": round(max(resize_ms), 3)}
+        st["e2e_tasks_per_s"] = round(n_tasks / r["wall_s"], 3)
+        if r["resize_ms"]:
+            rm = r["resize_ms"]
+            st["part_resize_ms"] = {"n": len(rm), **{k: round(v, 3) for k, v in percentiles(rm).items()},
+                                    "max": round(max(rm), 3)}
         out[label] = st
-        for p in parts:
-            mx.part_destroy(p)
     out["ratio_vs_1_partition"] = round(out["partitioned"]["tasks_per_s"]
                                         / out["1_partition"]["tasks_per_s"], 3)
     return out
