@@ -165,7 +165,8 @@ struct MpnnTrainParams {
   uint32_t off[11];          // element offsets of the 11 tensors in params (C1 ids)
   float* params;             // fp32 training state [n_params]
   float* partials;           // [n_tiles][n_params] per-tile gradients
-  float* hsave;              // [n_tiles][T+1][128][128] saved h^t (feature-major)
+  float* hsave;              // [n_tiles][T+5][128][128] saved h^t (feature-major) + backward scratch
+  uint8_t* wimg;             // mpnn_train_img_bytes(): tensor-core operand images of U, W_b
   const int* atom_off;
   const uint8_t* atom_type;
   const int* edge_off;
@@ -182,6 +183,7 @@ struct MpnnTrainParams {
 };
 int mpnn_train_smem_bytes();
 uint64_t mpnn_train_tile_scratch_floats(int T);
+uint64_t mpnn_train_img_bytes();
 int launch_mpnn_train(const MpnnTrainParams& p, void* stream);
 int launch_widen_bf16(float* dst, const uint16_t* src, uint64_t n, int n_ctas, void* stream);
 int mpnn_train_set_attrs(int device);

@@ -6,226 +6,262 @@
 //
 // Two launches per task on the partition's stream:
 //  1. mpnn_train_tile_kernel — one CTA per 128-atom tile (the inference
-//     kernel's packing): forward C4 keeping h^0..h^T (tile scratch in HBM),
-//     readout + loss terms, then the reverse-mode chain rule step by step
-//     (same order as oracle/mpnn_train.py), accumulating this tile's gradient
-//     of every parameter into its own partial buffer (no atomics).
+//     kernel's packing). Every [128 x 128] x [128 x 128] contraction runs on the
+//     5th-generation tensor cores (tcgen05.mma, fp32 accumulators in TMEM, one
+//     elected lane of warp 0 issues): the forward U h + sum_b W_b s_b with
+//     activations AND the fp32 parameters split into bf16 hi/lo terms (three
+//     products per K step, reading A17), then per step in reverse order
+//     dU^T = h^T-rows . dq-rows, dW_b^T = s_b^T-rows . dq-rows and
+//     dh = dq U + sum_b gather_b(dq) W_b with single bf16 terms (gradients are
+//     held to 2e-2, R10). Operands are staged in the K-major SWIZZLE_128B layout
+//     in whichever orientation makes the reduction index K (transposes happen
+//     while staging), h^0..h^T are kept in HBM scratch, the neighbour gathers
+//     and the readout / head run on the CUDA cores, and each weight gradient is
+//     drained from TMEM into this tile's partial (no atomics).
 //  2. mpnn_train_apply_kernel — every parameter element sums the tile
 //     partials in tile order (deterministic, independent of the partition
 //     size), applies the SGD update in place, and the loss is reduced in
 //     molecule order; the last CTA publishes the completion record.
-// Round-1 arithmetic is fp32 on CUDA cores (8x8 register blocks over
-// [128 x 128] shared-memory tiles); the tensor-core (tcgen05) version of the
-// backward contractions is the next step.
 #include "common.cuh"
 #include "kernels.h"
 #include "launch.cuh"
+#include "tc05.cuh"
 
 namespace mxk {
 
 namespace {
 constexpr int kF = 128;
-constexpr int kA = 128;            // atoms per tile
+constexpr int kA = 128;            // atoms per tile (MMA M / K over atoms)
 constexpr int kTE = 512;           // bonds per tile
-constexpr int kThreads = 256;
-constexpr int kS = 132;            // row stride (floats) of the [feature][atom] buffers
-constexpr int kBuf = kF * kS;      // floats per buffer
-constexpr int kWc = 16;            // weight rows per staged chunk
+constexpr int kThreads = 256;      // 8 warps: warp w drains TMEM lanes 32 (w % 4).., columns 64 (w / 4)..
+constexpr int kOp = kF * kA * 2;   // one [128][128] bf16 operand (two K-major SWIZZLE_128B halves)
+constexpr int kHalf = kOp / 2;
 
-// smem map (floats / ints)
-constexpr int kOffH = 0;
-constexpr int kOffS = kOffH + kBuf;
-constexpr int kOffD = kOffS + kBuf;
-constexpr int kOffW = kOffD + kBuf;                 // [kWc][kS] weight chunk
-constexpr int kOffNbrOff = kOffW + kWc * kS;        // int [kA + 4]
-constexpr int kOffNbr = kOffNbrOff + kA + 4;        // int [2 * kTE]: (u << 2) | b
-constexpr int kOffR = kOffNbr + 2 * kTE;            // float [kF] readout r
-constexpr int kOffZ = kOffR + kF;                   // float [kF] a (pre-activation)
-constexpr int kOffDA = kOffZ + kF;                  // float [kF] da
-constexpr int kOffDR = kOffDA + kF;                 // float [kF] dr
-constexpr int kOffRed = kOffDR + kF;                // float [16]
-constexpr int kOffOff4 = kOffRed + 16;              // int [kA][5]: per-bond-type neighbour ranges
-constexpr int kTrainSmem = (kOffOff4 + kA * 5) * 4;
-// setup-only aliases inside the S buffer (before the first neighbour gather)
-constexpr int kOffEdges = kOffS;                    // int4 [kTE]
-constexpr int kOffMolE = kOffS + 4 * kTE;           // int2 [kA]
+// smem map (bytes from a 1024-aligned base). Forward: H hi/lo, S hi/lo, W hi/lo.
+// Backward (single bf16 terms): dqT [f][v], dq [v][f], hT [k][v], X (sT_b [k][v]
+// or gq_b [v][f]), Wt [k][f] (U^T or W_b^T), h [v][k].
+constexpr int kOffOp0 = 0;                  // H hi | H lo      ; dqT | dq
+constexpr int kOffOp1 = kOffOp0 + 2 * kOp;  // S hi | S lo      ; hT  | X
+constexpr int kOffOp2 = kOffOp1 + 2 * kOp;  // W hi | W lo      ; Wt  | h
+constexpr int kOffNbrOff = kOffOp2 + 2 * kOp;       // int [kA + 4]
+constexpr int kOffNbr = kOffNbrOff + (kA + 4) * 4;  // int [2 * kTE]: (u << 2) | b
+constexpr int kOffOff4 = kOffNbr + 2 * kTE * 4;     // int [kA][5]: per-bond-type neighbour ranges
+constexpr int kOffRed = kOffOff4 + kA * 5 * 4;      // float [4][kF] column partials (dc) / head vectors
+constexpr int kOffVec = kOffRed + 4 * kF * 4;       // float [4][kF]: r, a, da, dr
+constexpr int kOffC = kOffVec + 4 * kF * 4;         // float [kF] bias c
+constexpr int kOffMisc = kOffC + kF * 4;            // float [16]
+constexpr int kOffBar = kOffMisc + 64;              // uint64 MMA-done mbarrier
+constexpr int kOffTmem = kOffBar + 8;               // uint32 TMEM base
+constexpr int kTrainSmem = kOffTmem + 8 + 1024;     // + alignment slack
+// setup-only aliases inside Op1 (before the first gather)
+constexpr int kOffEdges = kOffOp1;                  // int4 [kTE]
+constexpr int kOffMolE = kOffOp1 + 16 * kTE;        // int2 [kA]
+constexpr uint32_t kTmemCols = 256;                 // acc0: cols 0..127, acc1: cols 128..255
+constexpr uint32_t kIdesc = umma_idesc_bf16(128, 128);
 
-__device__ __forceinline__ float* fbuf(float* sm, int off) { return sm + off; }
+// 16-byte chunk ch (columns 8ch..8ch+7) of row `row` of a [128][128] operand
+__device__ __forceinline__ uint32_t chunk_off(int row, int ch) {
+  return (uint32_t)((ch >> 3) * kHalf + row * 128 + (((ch & 7) ^ (row & 7)) << 4));
+}
+__device__ __forceinline__ uint32_t elem_off(int row, int col) {
+  return chunk_off(row, col >> 3) + (col & 7) * 2;
+}
 
-// acc[i][j] (rows r = ta + 16 i of the OUTPUT's first index, cols c = tb + 16 j)
-struct Acc {
-  float v[8][8];
-  __device__ __forceinline__ void zero() {
+__device__ __forceinline__ uint4 pack8(const uint16_t (&v)[8]) {
+  return make_uint4(v[0] | ((uint32_t)v[1] << 16), v[2] | ((uint32_t)v[3] << 16),
+                    v[4] | ((uint32_t)v[5] << 16), v[6] | ((uint32_t)v[7] << 16));
+}
+// 8 fp32 -> bf16 hi (and lo = bf16(x - hi) if lo != nullptr) at operand chunk (row, ch)
+__device__ __forceinline__ void put8(uint8_t* hi, uint8_t* lo, int row, int ch, const float (&f)[8]) {
+  uint16_t h[8], l[8];
 #pragma unroll
-    for (int i = 0; i < 8; ++i)
-#pragma unroll
-      for (int j = 0; j < 8; ++j) v[i][j] = 0.f;
+  for (int j = 0; j < 8; ++j) {
+    h[j] = f32_to_bf16_rne(f[j]);
+    l[j] = f32_to_bf16_rne(f[j] - bf16_bits_to_f32(h[j]));
   }
-};
+  const uint32_t o = chunk_off(row, ch);
+  *reinterpret_cast<uint4*>(hi + o) = pack8(h);
+  if (lo) *reinterpret_cast<uint4*>(lo + o) = pack8(l);
+}
+__device__ __forceinline__ void get8(const uint8_t* op, int row, int ch, float (&f)[8]) {
+  unpack8(*reinterpret_cast<const uint4*>(op + chunk_off(row, ch)), f);
+}
 
-// G1: acc[v][f] += sum_k X[k][v] * W[f][k]   (X: smem [k][v]; W: global row-major [f][k])
-__device__ void gemm_xw_t(Acc& acc, const float* X, const float* __restrict__ W, float* Wt, int ta,
-                          int tb, int tid) {
-  for (int k0 = 0; k0 < kF; k0 += kWc) {
-    __syncthreads();
-    // Wt[kk][f] = W[f][k0 + kk]
-    for (int i = tid; i < kF * kWc; i += kThreads) {
-      const int f = i / kWc, kk = i - f * kWc;
-      Wt[kk * kS + f] = W[f * kF + k0 + kk];
+// Weight operand from fp32 parameters W[128][128] (row-major): rows r of the
+// operand = W rows (trans = 0) or W columns (trans = 1); hi (+ lo) bf16 terms.
+__device__ void stage_w(uint8_t* hi, uint8_t* lo, const float* __restrict__ W, bool trans, int tid) {
+  for (int i = tid; i < kF * 16; i += kThreads) {
+    const int r = i >> 4, ch = i & 15;
+    float f[8];
+    if (!trans) {
+      const float4 a = *reinterpret_cast<const float4*>(W + r * kF + 8 * ch);
+      const float4 b = *reinterpret_cast<const float4*>(W + r * kF + 8 * ch + 4);
+      f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+    } else {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) f[j] = W[(8 * ch + j) * kF + r];
     }
-    __syncthreads();
-#pragma unroll 4
-    for (int kk = 0; kk < kWc; ++kk) {
-      float x[8], w[8];
-#pragma unroll
-      for (int i = 0; i < 8; ++i) x[i] = X[(k0 + kk) * kS + ta + 16 * i];
-#pragma unroll
-      for (int j = 0; j < 8; ++j) w[j] = Wt[kk * kS + tb + 16 * j];
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 8; ++j) acc.v[i][j] = fmaf(x[i], w[j], acc.v[i][j]);
-    }
+    put8(hi, lo, r, ch, f);
   }
 }
 
-// G2: acc[v][k] += sum_f X[f][v] * W[f][k]   (X: smem [f][v]; W: global row-major [f][k])
-__device__ void gemm_xw(Acc& acc, const float* X, const float* __restrict__ W, float* Wc, int ta,
-                        int tb, int tid) {
-  for (int f0 = 0; f0 < kF; f0 += kWc) {
-    __syncthreads();
-    for (int i = tid; i < kWc * kF; i += kThreads) {
-      const int ff = i / kF, k = i - ff * kF;
-      Wc[ff * kS + k] = W[(f0 + ff) * kF + k];
-    }
-    __syncthreads();
-#pragma unroll 4
-    for (int ff = 0; ff < kWc; ++ff) {
-      float x[8], w[8];
+// out[v] = sum over the type-b neighbours u of v of src[u] (edge order), rows
+// of [128][128] operands (src hi (+ lo) summed); written as rows (trans = 0,
+// hi (+ lo)) or transposed as columns (trans = 1, hi only).
+__device__ void gather(uint8_t* out_hi, uint8_t* out_lo, const uint8_t* src_hi, const uint8_t* src_lo,
+                       const int* off4, const int* nbr, int na, int b, bool trans, int tid) {
+  for (int i = tid; i < kA * 16; i += kThreads) {
+    const int v = i >> 4, ch = i & 15;
+    const int q0 = (v < na) ? off4[v * 5 + b] : 0, q1 = (v < na) ? off4[v * 5 + b + 1] : 0;
+    float acc[8];
 #pragma unroll
-      for (int i = 0; i < 8; ++i) x[i] = X[(f0 + ff) * kS + ta + 16 * i];
+    for (int j = 0; j < 8; ++j) acc[j] = 0.f;
+    for (int q = q0; q < q1; ++q) {
+      const int u = nbr[q] >> 2;
+      float fh[8];
+      get8(src_hi, u, ch, fh);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) w[j] = Wc[ff * kS + tb + 16 * j];
+      for (int j = 0; j < 8; ++j) acc[j] += fh[j];
+      if (src_lo) {
+        float fl[8];
+        get8(src_lo, u, ch, fl);
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 8; ++j) acc.v[i][j] = fmaf(x[i], w[j], acc.v[i][j]);
-    }
-  }
-}
-
-// G3: G[f][k] += sum_v Z[f][v] * Y[k][v]  (both smem [.][v]); thread owns f = ta + 16 i,
-// k = tb + 16 j; accumulated into the tile's global gradient partial (owned, no atomics).
-__device__ void gemm_grad(float* __restrict__ G, const float* Z, const float* Y, int ta, int tb) {
-  Acc acc;
-  acc.zero();
-#pragma unroll 2
-  for (int v = 0; v < kA; v += 4) {
-    float4 z[8], y[8];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) z[i] = *reinterpret_cast<const float4*>(Z + (ta + 16 * i) * kS + v);
-#pragma unroll
-    for (int j = 0; j < 8; ++j) y[j] = *reinterpret_cast<const float4*>(Y + (tb + 16 * j) * kS + v);
-#pragma unroll
-    for (int i = 0; i < 8; ++i)
-#pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        float a = acc.v[i][j];
-        a = fmaf(z[i].x, y[j].x, a);
-        a = fmaf(z[i].y, y[j].y, a);
-        a = fmaf(z[i].z, y[j].z, a);
-        a = fmaf(z[i].w, y[j].w, a);
-        acc.v[i][j] = a;
+        for (int j = 0; j < 8; ++j) acc[j] += fl[j];
       }
-  }
+    }
+    if (!trans) {
+      put8(out_hi, out_lo, v, ch, acc);
+    } else {
 #pragma unroll
-  for (int i = 0; i < 8; ++i)
-#pragma unroll
-    for (int j = 0; j < 8; ++j) G[(ta + 16 * i) * kF + tb + 16 * j] += acc.v[i][j];
-}
-
-// S[k][v] = sum over the type-b neighbours u of v of X[k][u] (edge order). A
-// thread owns one atom v and half the features: its neighbour list is read
-// once (bucketed by bond type, off4[v][b] .. off4[v][b+1]) and reused for
-// every feature.
-constexpr int kGatherRegs = 8;
-__device__ void gather(float* S, const float* X, const int* off4, const int* nbr, int na, int b,
-                       int tid) {
-  const int v = tid % kA, k0 = tid / kA;
-  int u[kGatherRegs];
-  int q0 = 0, q1 = 0;
-  if (v < na) {
-    q0 = off4[v * 5 + b];
-    q1 = off4[v * 5 + b + 1];
-  }
-  const int c = q1 - q0;
-#pragma unroll
-  for (int q = 0; q < kGatherRegs; ++q) u[q] = (q < c) ? (nbr[q0 + q] >> 2) : 0;
-  for (int k = k0; k < kF; k += kThreads / kA) {
-    float t = 0.f;
-#pragma unroll
-    for (int q = 0; q < kGatherRegs; ++q)
-      if (q < c) t += X[k * kS + u[q]];
-    for (int q = q0 + kGatherRegs; q < q1; ++q) t += X[k * kS + (nbr[q] >> 2)];   // rare: deg > 8
-    S[k * kS + v] = t;
+      for (int j = 0; j < 8; ++j)
+        *reinterpret_cast<uint16_t*>(out_hi + elem_off(8 * ch + j, v)) = f32_to_bf16_rne(acc[j]);
+    }
   }
 }
 
-__device__ void save_buf(float* __restrict__ dst, const float* X, int tid) {
-  for (int i = tid; i < kF * kA / 4; i += kThreads) {
-    const int k = i / (kA / 4), v4 = (i - k * (kA / 4)) * 4;
-    *reinterpret_cast<float4*>(dst + k * kA + v4) = *reinterpret_cast<const float4*>(X + k * kS + v4);
+// Copy a precomputed operand image (global, L2-resident) into shared memory.
+__device__ __forceinline__ void copy_img(uint8_t* dst, const uint8_t* __restrict__ src, int bytes, int tid) {
+  for (int i = tid * 16; i < bytes; i += kThreads * 16)
+    *reinterpret_cast<uint4*>(dst + i) = *reinterpret_cast<const uint4*>(src + i);
+}
+// per matrix (U, W_0..W_3): forward image hi | lo ([f][k]) and backward image ([k][f], hi)
+constexpr int kImgBytes = 3 * kOp;
+
+// D (+)= A . B^T over K = 128 (8 MMAs of K = 16 per term pair), issued by warp 0
+// (warp-uniform descriptors, one elected lane), then committed to `bar`.
+__device__ __forceinline__ void mma_128(uint32_t d, uint32_t a, uint32_t b, bool accumulate) {
+#pragma unroll
+  for (int kk = 0; kk < kF / 16; ++kk) {
+    const uint32_t ko = (uint32_t)((kk >> 2) * kHalf + (kk & 3) * 32);
+    umma_f16_warp(d, umma_desc_sw128(a + ko), umma_desc_sw128(b + ko), kIdesc,
+                  (accumulate || kk > 0) ? 1u : 0u);
   }
 }
-__device__ void load_buf(float* X, const float* __restrict__ src, int tid) {
-  for (int i = tid; i < kF * kA / 4; i += kThreads) {
-    const int k = i / (kA / 4), v4 = (i - k * (kA / 4)) * 4;
-    *reinterpret_cast<float4*>(X + k * kS + v4) = *reinterpret_cast<const float4*>(src + k * kA + v4);
+
+// every thread: wait for the committed MMAs (phase parity `ph`, flipped after)
+__device__ __forceinline__ void mma_wait(uint64_t* bar, uint32_t& ph) {
+  while (!mbar_try_wait(bar, ph)) {
   }
+  __syncwarp();   // converged for the .sync.aligned tcgen05 loads that follow
+  ph ^= 1u;
+  tc_fence_after();
+}
+
+// This warp's 64 accumulator columns [c0, c0 + 64) of TMEM lane row (32 (w % 4) + lane).
+__device__ __forceinline__ void tmem_row64(uint32_t taddr, float (&v)[64]) {
+  uint32_t r[4][16];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) tmem_ld16_nowait(taddr + 16u * q, r[q]);
+  tmem_ld_wait();
+#pragma unroll
+  for (int q = 0; q < 4; ++q)
+#pragma unroll
+    for (int j = 0; j < 16; ++j) v[16 * q + j] = __uint_as_float(r[q][j]);
 }
 }  // namespace
 
 int mpnn_train_smem_bytes() { return kTrainSmem; }
-uint64_t mpnn_train_tile_scratch_floats(int T) { return (uint64_t)(T + 1) * kF * kA; }
+// per tile: h^0..h^T ([T+1][k][v]), dh^0 ([k][v]), per molecule (<= 128) dr, r, da ([m][k])
+uint64_t mpnn_train_tile_scratch_floats(int T) { return (uint64_t)(T + 5) * kF * kA; }
+uint64_t mpnn_train_img_bytes() { return 5ull * kImgBytes; }
+
+// Operand images of the task's fp32 parameters (the same for every tile):
+// U and W_b as forward B operands ([f][k], bf16 hi | lo) and backward B
+// operands ([k][f], bf16 hi), in the shared-memory layout, one CTA per matrix.
+__global__ void __launch_bounds__(kThreads) mpnn_train_prep_kernel(MpnnTrainParams p) {
+  const int m = blockIdx.x;   // 0 = U, 1 + b = W_b
+  if (m > p.n_bonds) return;
+  const float* W = p.params + (m == 0 ? p.off[5] : p.off[1] + (size_t)(m - 1) * kF * kF);
+  uint8_t* img = p.wimg + (size_t)m * kImgBytes;
+  stage_w(img, img + kOp, W, false, threadIdx.x);
+  stage_w(img + 2 * kOp, nullptr, W, true, threadIdx.x);
+}
 
 __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainParams p) {
-  extern __shared__ __align__(16) float sm[];
-  float* H = sm + kOffH;
-  float* S = sm + kOffS;
-  float* D = sm + kOffD;
-  float* Wst = sm + kOffW;
+  extern __shared__ __align__(1024) uint8_t smem_dyn[];
+  uint8_t* sm = smem_dyn + ((1024 - (smem_u32(smem_dyn) & 1023)) & 1023);
+  uint8_t* op0 = sm + kOffOp0;
+  uint8_t* op1 = sm + kOffOp1;
+  uint8_t* op2 = sm + kOffOp2;
   int* nbr_off = reinterpret_cast<int*>(sm + kOffNbrOff);
   int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
   int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
-  float* rr = sm + kOffR;
-  float* aa = sm + kOffZ;
-  float* da = sm + kOffDA;
-  float* dr = sm + kOffDR;
-  float* red = sm + kOffRed;
+  float* red = reinterpret_cast<float*>(sm + kOffRed);
+  float* rr = reinterpret_cast<float*>(sm + kOffVec);
+  float* aa = rr + kF;
+  float* da = aa + kF;
+  float* cvec = reinterpret_cast<float*>(sm + kOffC);
+  float* misc = reinterpret_cast<float*>(sm + kOffMisc);
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sm + kOffBar);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sm + kOffTmem);
   int4* ed = reinterpret_cast<int4*>(sm + kOffEdges);
   int2* mol_e = reinterpret_cast<int2*>(sm + kOffMolE);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int ta = tid >> 4, tb = tid & 15;
   const int F = kF;
   if (blockIdx.x == 0 && tid == 0) p.stamps[0] = globaltimer();
   const uint8_t* eb = reinterpret_cast<const uint8_t*>(p.edges);
   const float* E = p.params + p.off[0];
-  const float* Wb = p.params + p.off[1];
-  const float* U = p.params + p.off[5];
-  const float* cvec = p.params + p.off[6];
   const float* W1 = p.params + p.off[7];
   const float* c1 = p.params + p.off[8];
   const float* w2 = p.params + p.off[9];
   const float c2 = p.params[p.off[10]];
+  if (tid == 0) {
+    mbar_init(bar, 1);
+    fence_mbar_init();
+  }
+  if (warp == 0) tmem_alloc(tmem_slot, kTmemCols);
+  for (int i = tid; i < F; i += kThreads) cvec[i] = p.params[p.off[6] + i];
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = __shfl_sync(0xffffffffu, *tmem_slot, 0);
+  const uint32_t bar_s = smem_u32(bar);
+  uint32_t ph = 0;
+  const uint32_t s0 = smem_u32(op0), s1 = smem_u32(op1), s2 = smem_u32(op2);
+  const uint32_t acc0 = tmem, acc1 = tmem + 128u;
+  // this thread's TMEM row (lane) and column half
+  const int trow = 32 * (warp & 3) + lane, tc0 = 64 * (warp >> 2);
+  const uint32_t lane_off = (uint32_t)(32 * (warp & 3)) << 16;
 
   for (int tile = blockIdx.x; tile < p.n_tiles; tile += p.n_ctas) {
     float* G = p.partials + (uint64_t)tile * p.n_params;
-    float* hs = p.hsave + (uint64_t)tile * (p.T + 1) * kF * kA;
+    float* hs = p.hsave + (uint64_t)tile * (p.T + 5) * kF * kA;   // [T+1][k][v]
+    float* dh0 = hs + (uint64_t)(p.T + 1) * kF * kA;               // [k][v]
+    float* drm = dh0 + (uint64_t)kF * kA;                          // [molecule][k]
+    float* rm = drm + (uint64_t)kF * kA;                           // [molecule][k]
+    float* dam = rm + (uint64_t)kF * kA;                           // [molecule][f]
     const int m0 = p.tile_off[tile], m1 = p.tile_off[tile + 1];
     const int a0 = p.atom_off[m0], na = p.atom_off[m1] - a0;
     const int e0 = p.edge_off[m0], ne = p.edge_off[m1] - e0;
-    // zero this tile's gradient partial
-    for (int i = tid; i < p.n_params; i += kThreads) G[i] = 0.f;
+    {
+      // zero this tile's partial except U and the W_b the backward writes whole
+      // (W_b of bond types absent from the tile stay zero)
+      for (int i = tid; i < p.n_params; i += kThreads) {
+        const bool u_or_w = (i >= (int)p.off[1] && i < (int)p.off[1] + 4 * F * F) ||
+                            (i >= (int)p.off[5] && i < (int)p.off[5] + F * F);
+        if (!u_or_w) G[i] = 0.f;
+      }
+    }
     // --- tile CSR (as the inference kernel): edges in tile-local atom ids --------
     for (int i = tid; i < kA; i += kThreads) mol_e[i] = make_int2(0, 0);
     __syncthreads();
@@ -300,42 +336,71 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
     __syncthreads();
     int present = 0;
     for (int q = 0; q < nbr_off[kA]; ++q) present |= 1 << (nbr[q] & 3);
-    // --- forward: h^0 = E[type], h^{t+1} = ReLU(U h + sum_b W_b s_b + c) ------
-    for (int i = tid; i < F * kA; i += kThreads) {
-      const int k = i / kA, v = i - k * kA;
-      H[k * kS + v] = (v < na) ? E[(int)p.atom_type[a0 + v] * F + k] : 0.f;
+    for (int b = 0; b < 4; ++b)   // absent bond types: zero gradient partial
+      if (!(present & (1 << b)))
+        for (int i = tid; i < F * F; i += kThreads) G[p.off[1] + (size_t)b * F * F + i] = 0.f;
+    // ===================== forward (C4), h^{t+1} = ReLU(U h + sum_b W_b s_b + c) ===
+    for (int i = tid; i < kA * 16; i += kThreads) {
+      const int v = i >> 4, ch = i & 15;
+      float f[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        f[j] = (v < na) ? E[(int)p.atom_type[a0 + v] * F + 8 * ch + j] : 0.f;
+      put8(op0, op0 + kOp, v, ch, f);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) hs[(8 * ch + j) * kA + v] = f[j];
+    }
+    for (int t = 0; t < p.T; ++t) {
+      bool first = true;
+      for (int b = -1; b < p.n_bonds; ++b) {
+        if (b >= 0 && !(present & (1 << b))) continue;
+        // operands: A = H (b = -1) or S_b, B = U or W_b, both hi/lo (3 products)
+        __syncthreads();   // previous MMAs done (waited) -> S / W buffers free
+        if (b >= 0) gather(op1, op1 + kOp, op0, op0 + kOp, off4, nbr, na, b, false, tid);
+        copy_img(op2, p.wimg + (size_t)(b + 1) * kImgBytes, 2 * kOp, tid);   // W (hi | lo)
+        fence_proxy_async();
+        tc_fence_before();
+        __syncthreads();
+        if (warp == 0) {
+          tc_fence_after();
+          const uint32_t a = b < 0 ? s0 : s1;
+          mma_128(acc0, a, s2, !first);                  // A_hi . W_hi
+          mma_128(acc0, a + kOp, s2, true);              // A_lo . W_hi
+          mma_128(acc0, a, s2 + kOp, true);              // A_hi . W_lo
+          umma_commit_warp(bar_s);
+        }
+        mma_wait(bar, ph);
+        first = false;
+      }
+      // epilogue: h = ReLU(acc + c) -> H (hi/lo) and hs[t+1] ([k][v], fp32)
+      {
+        float v64[64];
+        tmem_row64(acc0 + lane_off + (uint32_t)tc0, v64);
+        tc_fence_before();
+        __syncthreads();   // every warp read its accumulator rows before H is overwritten
+        const int v = trow;
+        float* hn = hs + (size_t)(t + 1) * F * kA;
+#pragma unroll
+        for (int c8 = 0; c8 < 8; ++c8) {
+          float o[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const int f = tc0 + 8 * c8 + j;
+            o[j] = (v < na) ? fmaxf(v64[8 * c8 + j] + cvec[f], 0.f) : 0.f;
+            hn[f * kA + v] = o[j];
+          }
+          put8(op0, op0 + kOp, v, (tc0 >> 3) + c8, o);
+        }
+      }
     }
     __syncthreads();
-    save_buf(hs, H, tid);
-    for (int t = 0; t < p.T; ++t) {
-      Acc acc;
-      acc.zero();
-      gemm_xw_t(acc, H, U, Wst, ta, tb, tid);
-      for (int b = 0; b < p.n_bonds; ++b) {
-        if (!(present & (1 << b))) continue;
-        __syncthreads();
-        gather(S, H, off4, nbr, na, b, tid);
-        gemm_xw_t(acc, S, Wb + (size_t)b * F * F, Wst, ta, tb, tid);   // syncs before reading S
-      }
-      __syncthreads();
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int v = ta + 16 * i, f = tb + 16 * j;
-          H[f * kS + v] = (v < na) ? fmaxf(acc.v[i][j] + cvec[f], 0.f) : 0.f;
-        }
-      __syncthreads();
-      save_buf(hs + (size_t)(t + 1) * F * kA, H, tid);
-    }
-    // --- readout, loss term, head gradients, dh^T (per molecule, atom order) --
-    for (int i = tid; i < F * kA; i += kThreads) D[(i / kA) * kS + (i % kA)] = 0.f;
+    // ===================== readout, loss, head gradients (per molecule) ==========
+    const float* hT = hs + (size_t)p.T * F * kA;
     for (int m = m0; m < m1; ++m) {
       const int ab = p.atom_off[m] - a0, ae = p.atom_off[m + 1] - a0;
-      __syncthreads();
       if (tid < F) {
         float r = 0.f;
-        for (int v = ab; v < ae; ++v) r += H[tid * kS + v];
+        for (int v = ab; v < ae; ++v) r += hT[tid * kA + v];
         rr[tid] = r;
       }
       __syncthreads();
@@ -345,7 +410,6 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         aa[tid] = a;
       }
       __syncthreads();
-      // y = w2 . ReLU(a) + c2 (warp 0, fixed shuffle tree)
       if (warp == 0) {
         float part = 0.f;
         for (int f = lane; f < F; f += 32) part = fmaf(w2[f], fmaxf(aa[f], 0.f), part);
@@ -354,80 +418,169 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
           const float y = part + c2;
           p.y[m] = y;
           p.out[m] = y;
-          red[8] = 2.0f * (y - p.targets[m]) / (float)p.n_mol;   // dy
+          misc[0] = 2.0f * (y - p.targets[m]) / (float)p.n_mol;   // dy
         }
       }
       __syncthreads();
-      const float dy = red[8];
+      const float dy = misc[0];
       if (tid < F) {
-        const float z = fmaxf(aa[tid], 0.f);
-        G[p.off[9] + tid] += dy * z;                               // dw2
-        const float d = (aa[tid] > 0.f) ? dy * w2[tid] : 0.f;      // da
+        G[p.off[9] + tid] += dy * fmaxf(aa[tid], 0.f);              // dw2
+        const float d = (aa[tid] > 0.f) ? dy * w2[tid] : 0.f;        // da
         da[tid] = d;
-        G[p.off[8] + tid] += d;                                    // dc1
+        G[p.off[8] + tid] += d;                                      // dc1
       }
-      if (tid == 0) G[p.off[10]] += dy;                            // dc2
+      if (tid == 0) G[p.off[10]] += dy;                              // dc2
+      if (tid < F) {
+        rm[(m - m0) * F + tid] = rr[tid];
+        dam[(m - m0) * F + tid] = da[tid];
+      }
       __syncthreads();
-      // dW1 += da r^T ; dr = W1^T da
-      for (int i = tid; i < F * F; i += kThreads) {
-        const int f = i / F, k = i - f * F;
-        G[p.off[7] + i] += da[f] * rr[k];
-      }
       if (tid < F) {
         float s = 0.f;
         for (int f = 0; f < F; ++f) s = fmaf(W1[f * F + tid], da[f], s);
-        dr[tid] = s;
+        drm[(m - m0) * F + tid] = s;                                 // dr: dh^T of every atom of m
       }
       __syncthreads();
-      for (int i = tid; i < F * (ae - ab); i += kThreads) {
-        const int k = i / (ae - ab), v = ab + (i - k * (ae - ab));
-        D[k * kS + v] = dr[k];
-      }
     }
-    __syncthreads();
-    // --- backward through the T message-passing steps --------------------------
+    // dW1 += sum_m da_m r_m^T (molecule order, one pass over the partial)
+    for (int i = tid; i < F * F; i += kThreads) {
+      const int f = i / F, k = i - f * F;
+      float g = 0.f;
+      for (int m = 0; m < m1 - m0; ++m) g = fmaf(dam[m * F + f], rm[m * F + k], g);
+      G[p.off[7] + i] += g;
+    }
+    // ===================== backward through the T message-passing steps ==========
+    // per step (reverse): dq = dh * [h^{t+1} > 0]; dc += sum_v dq; dU += dq^T h;
+    // dW_b += dq^T s_b; dh^t = dq U + sum_b gather_b(dq) W_b
+    uint8_t* dqT = op0;            // [f][v]  (B of the weight gradients)
+    uint8_t* dq = op0 + kOp;       // [v][f]  (A of dh)
+    uint8_t* hTo = op1;            // [k][v]  (A of dU)
+    uint8_t* X = op1 + kOp;        // sT_b [k][v] (A of dW_b) / gq_b [v][f] (A of dh)
+    uint8_t* Wt = op2;             // [k][f]  (B of dh)
+    uint8_t* hv = op2 + kOp;       // [v][k]  (gather source for s_b)
+    const uint32_t sdqT = s0, sdq = s0 + kOp, shT = s1, sX = s1 + kOp, sWt = s2;
     for (int t = p.T - 1; t >= 0; --t) {
-      const float* hn = hs + (size_t)(t + 1) * F * kA;
-      // dq = dh^{t+1} * [h^{t+1} > 0]   (in place in D)
-      for (int i = tid; i < F * kA; i += kThreads) {
-        const int k = i / kA, v = i - k * kA;
-        if (!(hn[k * kA + v] > 0.f)) D[k * kS + v] = 0.f;
+      // (a) dq from dh (acc1, or the readout's dr at the last step) and the mask
+      {
+        float dh64[64];
+        const int v = trow;
+        if (t == p.T - 1) {
+          int ml = 0;   // v's molecule (tile-local)
+          while (ml + 1 < m1 - m0 && p.atom_off[m0 + ml + 1] - a0 <= v) ++ml;
+#pragma unroll
+          for (int j = 0; j < 64; ++j) dh64[j] = (v < na) ? drm[ml * F + tc0 + j] : 0.f;
+        } else {
+          tmem_row64(acc1 + lane_off + (uint32_t)tc0, dh64);
+        }
+        tc_fence_before();
+        __syncthreads();   // acc1 read everywhere; operands of step t+1 free
+        const float* hn = hs + (size_t)(t + 1) * F * kA;
+#pragma unroll
+        for (int c8 = 0; c8 < 8; ++c8) {
+          float o[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const int f = tc0 + 8 * c8 + j;
+            o[j] = (v < na && hn[f * kA + v] > 0.f) ? dh64[8 * c8 + j] : 0.f;
+            *reinterpret_cast<uint16_t*>(dqT + elem_off(f, v)) = f32_to_bf16_rne(o[j]);
+            // dc: column sums over this warp's 32 rows (fixed shuffle tree)
+            const float cs = warp_sum(o[j]);
+            if (lane == 0) red[(warp & 3) * F + f] = cs;
+          }
+          put8(dq, nullptr, v, (tc0 >> 3) + c8, o);
+        }
       }
-      load_buf(H, hs + (size_t)t * F * kA, tid);
+      // (b) h^t as hT [k][v] and h [v][k] (bf16) from the saved fp32 rows
+      {
+        const float* ht = hs + (size_t)t * F * kA;
+        for (int i = tid; i < kF * 16; i += kThreads) {
+          const int k = i >> 4, ch = i & 15;
+          float f[8];
+          const float4 a4 = *reinterpret_cast<const float4*>(ht + k * kA + 8 * ch);
+          const float4 b4 = *reinterpret_cast<const float4*>(ht + k * kA + 8 * ch + 4);
+          f[0] = a4.x; f[1] = a4.y; f[2] = a4.z; f[3] = a4.w; f[4] = b4.x; f[5] = b4.y; f[6] = b4.z; f[7] = b4.w;
+          put8(hTo, nullptr, k, ch, f);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            *reinterpret_cast<uint16_t*>(hv + elem_off(8 * ch + j, k)) = f32_to_bf16_rne(f[j]);
+        }
+      }
+      copy_img(Wt, p.wimg + 2 * kOp, kOp, tid);                     // U^T
+      fence_proxy_async();
+      tc_fence_before();
       __syncthreads();
-      if (tid < F) {
-        float s = 0.f;
-        for (int v = 0; v < na; ++v) s += D[tid * kS + v];
-        G[p.off[6] + tid] += s;                                    // dc
+      if (tid < F) G[p.off[6] + tid] += (red[tid] + red[F + tid]) + (red[2 * F + tid] + red[3 * F + tid]);   // dc
+      if (warp == 0) {
+        tc_fence_after();
+        mma_128(acc0, shT, sdqT, false);     // dU^T[k][f] = sum_v h[v][k] dq[v][f]
+        mma_128(acc1, sdq, sWt, false);      // dh[v][k]   = sum_f dq[v][f] U[f][k]
+        umma_commit_warp(bar_s);
       }
-      gemm_grad(G + p.off[5], D, H, ta, tb);                       // dU += dq^T h
-      Acc acc;
-      acc.zero();
-      gemm_xw(acc, D, U, Wst, ta, tb, tid);                        // dh = dq U
+      mma_wait(bar, ph);
+      // flush a weight gradient (acc0 = [k][f]) into this tile's partial G[f][k]
+      // (the partial of U / W_b is written by the first backward step, t = T-1)
+      auto flush = [&](float* Gm, bool set) {
+        float g64[64];
+        tmem_row64(acc0 + lane_off + (uint32_t)tc0, g64);
+        const int k = trow;
+        if (set) {
+#pragma unroll
+          for (int j = 0; j < 64; ++j) Gm[(tc0 + j) * F + k] = g64[j];
+        } else {
+#pragma unroll
+          for (int j = 0; j < 64; ++j) Gm[(tc0 + j) * F + k] += g64[j];
+        }
+      };
+      flush(G + p.off[5], t == p.T - 1);                            // dU
       for (int b = 0; b < p.n_bonds; ++b) {
         if (!(present & (1 << b))) continue;
+        tc_fence_before();
+        __syncthreads();   // acc0 flushed, X free
+        gather(X, nullptr, hv, nullptr, off4, nbr, na, b, true, tid);   // sT_b [k][v]
+        fence_proxy_async();
+        tc_fence_before();
         __syncthreads();
-        gather(S, H, off4, nbr, na, b, tid);                    // s_b(h^t)
-        __syncthreads();
-        gemm_grad(G + p.off[1] + (size_t)b * F * F, D, S, ta, tb); // dW_b += dq^T s_b
-        __syncthreads();
-        gather(S, D, off4, nbr, na, b, tid);                    // sum of neighbours' dq
-        gemm_xw(acc, S, Wb + (size_t)b * F * F, Wst, ta, tb, tid); // dh += (.) W_b
-      }
-      __syncthreads();
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const int v = ta + 16 * i, k = tb + 16 * j;
-          D[k * kS + v] = (v < na) ? acc.v[i][j] : 0.f;
+        if (warp == 0) {
+          tc_fence_after();
+          mma_128(acc0, sX, sdqT, false);    // dW_b^T[k][f] = sum_v s_b[v][k] dq[v][f]
+          umma_commit_warp(bar_s);
         }
+        mma_wait(bar, ph);
+        flush(G + p.off[1] + (size_t)b * F * F, t == p.T - 1);      // dW_b
+        tc_fence_before();
+        __syncthreads();   // X and Wt free
+        gather(X, nullptr, dq, nullptr, off4, nbr, na, b, false, tid);  // gq_b [v][f]
+        copy_img(Wt, p.wimg + (size_t)(b + 1) * kImgBytes + 2 * kOp, kOp, tid);   // W_b^T
+        fence_proxy_async();
+        tc_fence_before();
+        __syncthreads();
+        if (warp == 0) {
+          tc_fence_after();
+          mma_128(acc1, sX, sWt, true);      // dh[v][k] += sum_f gq_b[v][f] W_b[f][k]
+          umma_commit_warp(bar_s);
+        }
+        mma_wait(bar, ph);
+      }
+      tc_fence_before();
       __syncthreads();
     }
-    // dE[type_v] += dh^0_v (atom order)
-    if (tid < F)
-      for (int v = 0; v < na; ++v) G[p.off[0] + (int)p.atom_type[a0 + v] * F + tid] += D[tid * kS + v];
+    // dE[type_v] += dh^0_v (atom order): dh^0 ([k][v], fp32) through the scratch
+    {
+      float dh64[64];
+      tmem_row64(acc1 + lane_off + (uint32_t)tc0, dh64);
+      const int v = trow;
+#pragma unroll
+      for (int j = 0; j < 64; ++j) dh0[(tc0 + j) * kA + v] = (v < na) ? dh64[j] : 0.f;
+    }
     __syncthreads();
+    if (tid < F)
+      for (int v = 0; v < na; ++v) G[p.off[0] + (int)p.atom_type[a0 + v] * F + tid] += dh0[tid * kA + v];
+    tc_fence_before();
+    __syncthreads();
+  }
+  if (warp == 0) {
+    tc_fence_after();
+    tmem_dealloc(tmem, kTmemCols);
   }
 }
 
@@ -476,8 +629,10 @@ __global__ void widen_bf16_kernel(float* dst, const uint16_t* src, uint64_t n) {
 int launch_mpnn_train(const MpnnTrainParams& p, void* stream) {
   MpnnTrainParams pc = p;
   void* args[] = {&pc};
-  int rc = launch_kernel(mpnn_train_tile_kernel, dim3(p.n_ctas), dim3(kThreads),
-                         (unsigned)kTrainSmem, stream, args);
+  int rc = launch_kernel(mpnn_train_prep_kernel, dim3(1 + p.n_bonds), dim3(kThreads), 0u, stream, args);
+  if (rc) return rc;
+  rc = launch_kernel(mpnn_train_tile_kernel, dim3(p.n_ctas), dim3(kThreads),
+                     (unsigned)kTrainSmem, stream, args);
   if (rc) return rc;
   return launch_kernel(mpnn_train_apply_kernel, dim3(p.n_ctas), dim3(kThreads), 0u, stream, args);
 }

@@ -92,7 +92,7 @@ struct Slot {
   // mpnn: device image of a task's packed inputs (Task::blob)
   CUdeviceptr in_blob = 0;
   // mpnn training (N4)
-  CUdeviceptr y = 0, partials = 0, hsave = 0;
+  CUdeviceptr y = 0, partials = 0, hsave = 0, wimg = 0;
   // common
   CUdeviceptr bar = 0, stamps = 0, err = 0;
   uint64_t bar_count = 0;
