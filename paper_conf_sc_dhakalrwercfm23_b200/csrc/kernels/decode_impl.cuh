@@ -174,15 +174,20 @@ struct Smem {
 };
 
 template <int B>
-__device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax) {
+__device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax, int fuse_att) {
   Smem s;
   uint8_t* p = raw + ((1024 - (smem_u32(raw) & 1023)) & 1023);
   s.ring = p;
   p += (size_t)n_stages * kStageBytes;
   s.act = p;
   p += (size_t)decode_act_bytes(B, kmax);
-  s.att = reinterpret_cast<float*>(p);
-  p += (size_t)kConsumerWarps * 3 * kAttHd * 4;
+  if (decode_att_in_act(B, kmax, fuse_att)) {
+    // separate attention phase: the operand is idle while attention runs
+    s.att = reinterpret_cast<float*>(s.act);
+  } else {
+    s.att = reinterpret_cast<float*>(p);
+    p += (size_t)kConsumerWarps * 3 * kAttHd * 4;
+  }
   s.full = reinterpret_cast<uint64_t*>(p);
   p += (size_t)n_stages * 8;
   s.empty = reinterpret_cast<uint64_t*>(p);
@@ -932,7 +937,7 @@ template <int B>
 __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams p, int n_stages,
                                                                    int kmax) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  const Smem sm = carve<B>(smem_raw, n_stages, kmax);
+  const Smem sm = carve<B>(smem_raw, n_stages, kmax, p.fuse_att);
   const int warp_id = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < n_stages; ++i) {
@@ -1060,7 +1065,7 @@ template <int B>
 int launch_b(const DecodeParams& p, void* stream, int cooperative) {
   const int kmax = max(max(p.d, p.q_dim), p.ff);
   int ns = 0;
-  const int smem = decode_smem_bytes(B, kmax, &ns);
+  const int smem = decode_smem_bytes(B, kmax, &ns, p.fuse_att);
   if (smem < 0) return -3;
   DecodeParams pc = p;
   int ns_arg = ns, kmax_arg = kmax;

@@ -111,8 +111,13 @@ int decode_prof_buckets();
 // Number of grid barriers one decode launch performs (host bookkeeping of bar_base).
 uint64_t decode_barriers(int L, int P, int G, int fuse_att);
 
-// Shared-memory bytes of the decode kernel for a given shape (-1: does not fit).
-int decode_smem_bytes(int B, int kmax, int* n_stages);
+// Shared-memory bytes of the decode kernel for a given shape (-1: does not fit);
+// fuse_att = 0 (separate attention phase) lets the attention scratch share the
+// activation operand, leaving more of the 227 KiB to the weight ring.
+int decode_smem_bytes(int B, int kmax, int* n_stages, int fuse_att = 1);
+MX_HD constexpr bool decode_att_in_act(int B, int kmax, int fuse_att) {
+  return !fuse_att && decode_act_bytes(B, kmax) >= kConsumerWarps * 3 * kAttHd * 4;
+}
 
 // cooperative != 0: cuLaunchCooperativeKernel (all CTAs co-resident; used on
 // unpartitioned streams where other kernels compete for the same SMs).
