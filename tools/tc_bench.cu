@@ -94,6 +94,37 @@ __global__ void bench(int M, int N, int iters, int a_boxes, int accs, int warp_w
       out[0] = c1 - c0;
       out[1] = c2 - c0;
     }
+  } else if (warp_wide == 3 && threadIdx.x < 64) {
+    // two warps issue concurrently into disjoint accumulators (uniform descriptors)
+    const int w = threadIdx.x >> 5;
+    const uint32_t id = idesc(M, N);
+    const uint32_t tu = __shfl_sync(0xffffffffu, t, 0) + (uint32_t)(w * 128);
+    const uint64_t ad0 = desc_sw128(su32(base) + w * 65536, 1024), bd0 = desc_sw128(su32(base + 128 * 1024), 1024);
+    __syncwarp();
+    long long c0 = clock64();
+    for (int i = 0; i < iters / 8; ++i) {
+      const int box = i % 4;
+      const uint64_t ad = ad0 + (uint64_t)(box * 1024), bd = bd0 + (uint64_t)((box & 3) * 128);
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        asm volatile("{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                     "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tu),
+                     "l"(ad + 2 * j), "l"(bd + 2 * j), "r"(id), "r"((i | j) ? 1 : 0));
+    }
+    long long c1 = clock64();
+    if (w == 0) {
+      asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+                   "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(&bar)));
+      uint32_t ok = 0;
+      while (!ok)
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok) : "r"(su32(&bar)));
+      long long c2 = clock64();
+      if (threadIdx.x == 0) {
+        out[0] = c1 - c0;
+        out[1] = c2 - c0;
+      }
+    }
   } else if (threadIdx.x == 0 && !warp_wide) {
     const uint32_t id = idesc(M, N);
     const uint32_t a0 = su32(base), b0 = su32(base + 128 * 1024);
@@ -140,6 +171,8 @@ int main() {
       {128, 64, 8, 1, 2, "uniform descs: M128 N64"},
       {128, 256, 8, 1, 2, "uniform descs: M128 N256"},
       {64, 16, 8, 1, 2, "uniform descs: M64 N16"},
+      {128, 16, 8, 1, 3, "2 warps concurrently, M128 N16 (per MMA of all)"},
+      {64, 16, 8, 1, 3, "2 warps concurrently, M64 N16 (per MMA of all)"},
   };
   for (auto& c : cfgs) {
     const int iters = 4096;

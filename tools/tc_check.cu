@@ -14,6 +14,7 @@ __device__ __forceinline__ uint64_t desc_sw128(uint32_t saddr, uint32_t sbo) {
          ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(16 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+constexpr uint32_t kIdesc64 = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(16 >> 3) << 17) | ((uint32_t)(64 >> 4) << 24);
 
 // element (row, k) of a [rows][64] K-major SW128 operand
 __device__ __forceinline__ uint32_t off(int row, int k) {
@@ -60,6 +61,13 @@ __global__ void check(const float* A, const float* Bm, float* D, int mode, uint3
                    "l"(ad + 2 * j), "l"(bd + 2 * j), "r"(kIdesc), "r"(j > 0 ? 1 : 0));
     asm volatile("{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
                  "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(su32(&bar)));
+  } else if (mode == 3 && tid == 0) {
+    // M = 64: where do the 64 rows of D land in TMEM?
+    for (int j = 0; j < 4; ++j)
+      asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                   "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(t),
+                   "l"(ad + 2 * j), "l"(bd + 2 * j), "r"(kIdesc64), "r"(j > 0 ? 1 : 0));
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(su32(&bar)));
   } else if (mode == 2 && tid < 32) {
     const uint32_t tu = __shfl_sync(0xffffffffu, t, 0);
     for (int j = 0; j < 4; ++j)
@@ -97,6 +105,28 @@ int main() {
   cudaMemcpy(A, hA, sizeof hA, cudaMemcpyHostToDevice);
   cudaMemcpy(Bm, hB, sizeof hB, cudaMemcpyHostToDevice);
   cudaFuncSetAttribute(check, cudaFuncAttributeMaxDynamicSharedMemorySize, 40 * 1024);
+  {
+    // M = 64 layout probe: for each TMEM lane, which row m of D (if any) it holds
+    cudaMemset(D, 0, sizeof hD);
+    check<<<1, 128, 40 * 1024>>>(A, Bm, D, 3, 1024);
+    cudaDeviceSynchronize();
+    cudaMemcpy(hD, D, sizeof hD, cudaMemcpyDeviceToHost);
+    printf("M=64 lane -> row:");
+    for (int lane = 0; lane < 128; ++lane) {
+      int found = -1;
+      for (int m = 0; m < 64 && found < 0; ++m) {
+        bool ok = true;
+        for (int n = 0; n < 16 && ok; ++n) {
+          double ref = 0;
+          for (int k = 0; k < 64; ++k) ref += (double)hA[m * 64 + k] * hB[n * 64 + k];
+          ok = fabs(ref - hD[lane * 16 + n]) < 1e-3;
+        }
+        if (ok) found = m;
+      }
+      printf(" %d:%d", lane, found);
+    }
+    printf("\n");
+  }
   for (int sbo = 0; sbo <= 1024; sbo += 1024)
     for (int mode = 0; mode < 3; ++mode) {
       cudaMemset(D, 0, sizeof hD);
