@@ -224,6 +224,10 @@ def choose_layout(mx, fn, args, sweep, prompts):
 def gpu_arm(args, rank, world, local_rank, dist):
     from paper_conf_sc_dhakalrwercfm23_b200 import mx
     devices = local_devices(args.gpus, world, local_rank)
+    if args.devices:
+        # explicit device list for this process (e.g. "0,0": the in-process
+        # multi-GPU path on one physical device — two dispatchers, one placement)
+        devices = [int(x) for x in args.devices.split(",")]
     mx.mx_init(devices)
     gpus = list(range(len(devices)))          # library GPU indices
     ng = len(gpus)
@@ -539,6 +543,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="mx", choices=["mx", "reference"])
+    ap.add_argument("--devices", default="",
+                    help="explicit device ordinals for this process (default: --gpus / LOCAL_RANK)")
     ap.add_argument("--layout", default="auto")
     ap.add_argument("--sweep", default="1,2,4,7,14,18,37",
                     help="comma list of partition counts for the pre-run sweep ('' = none)")
