@@ -366,7 +366,9 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
         if (si + 1 < nseg) nxt = p.w_b + (size_t)(seg_list[si + 1] - 1) * kF * kF;
         else if (step + 1 < p.T) nxt = p.u;
         else nxt = p.w1;   // readout weights, prefetched under the last MMA
-        if (tid == 0) {
+        if (warp == 0) {
+          // warp-uniform issue, one elected lane (tc05.cuh: ~2-3x the issue rate of
+          // a single divergent thread)
           tc_fence_after();
           const uint32_t a_hi = seg > 0 ? Shi : Hhi, a_lo = seg > 0 ? Slo : Hlo;
           const uint32_t w = Wbuf[wi];
@@ -374,10 +376,10 @@ __global__ void __launch_bounds__(kMpnnThreads, 1) mpnn_kernel(MpnnParams p) {
           for (int kk = 0; kk < kF / 16; ++kk) {
             const uint32_t koff = (uint32_t)((kk >> 2) * kHalfBytes + (kk & 3) * 32);
             const uint64_t bdesc = umma_desc_sw128(w + koff);
-            umma_bf16(tmem, umma_desc_sw128(a_hi + koff), bdesc, (si > 0 || kk > 0) ? 1u : 0u);
-            umma_bf16(tmem, umma_desc_sw128(a_lo + koff), bdesc, 1u);
+            umma_f16_warp(tmem, umma_desc_sw128(a_hi + koff), bdesc, kIdesc, (si > 0 || kk > 0) ? 1u : 0u);
+            umma_f16_warp(tmem, umma_desc_sw128(a_lo + koff), bdesc, kIdesc, 1u);
           }
-          umma_commit(bar_s);                  // arrives when these MMAs have completed
+          umma_commit_warp(bar_s);             // arrives when these MMAs have completed
         }
         if (nxt) load_matrix_async(Wbuf[wi ^ 1], nxt, tid);
         // the U.h contraction does not read S: build the next neighbour sum under it
