@@ -125,6 +125,40 @@ __global__ void bench(int M, int N, int iters, int a_boxes, int accs, int warp_w
         out[1] = c2 - c0;
       }
     }
+  } else if ((warp_wide == 4 || warp_wide == 5) && threadIdx.x < 32) {
+    // per-box mbarrier wait inside the loop (the barrier is already complete):
+    // 4 = C++ polling loop + __syncwarp (as the decode kernel), 5 = spin loop inside PTX
+    const uint32_t id = idesc(M, N);
+    const uint32_t tu = __shfl_sync(0xffffffffu, t, 0);
+    const uint32_t a0 = su32(base), b0 = su32(base + 128 * 1024);
+    const uint32_t wb = su32(&bar);
+    long long c0 = clock64();
+    uint32_t stage = 0;
+    for (int i = 0; i < iters / 4; ++i) {
+      if (warp_wide == 4) {
+        uint32_t ok = 0;
+        while (!ok)
+          asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], 1;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                       : "=r"(ok) : "r"(wb));
+        __syncwarp();
+      } else {
+        asm volatile("{\n\t.reg .pred p;\n\tWAIT_%=:\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%0], 1;\n\t@!p bra WAIT_%=;\n\t}" ::"r"(wb) : "memory");
+      }
+      const uint32_t sa = a0 + stage * 16384u;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const uint64_t ad = desc_sw128(sa + j * 32, 1024), bd = desc_sw128(b0 + j * 32, 1024);
+        asm volatile("{\n\t.reg .pred e, p;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+                     "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tu),
+                     "l"(ad), "l"(bd), "r"(id), "r"((i | j) ? 1 : 0));
+      }
+      if (++stage == (uint32_t)a_boxes) stage = 0;
+    }
+    long long c1 = clock64();
+    if (threadIdx.x == 0) {
+      out[0] = c1 - c0;
+      out[1] = c1 - c0;
+    }
   } else if (threadIdx.x == 0 && !warp_wide) {
     const uint32_t id = idesc(M, N);
     const uint32_t a0 = su32(base), b0 = su32(base + 128 * 1024);
@@ -172,6 +206,8 @@ int main() {
       {128, 256, 8, 1, 2, "uniform descs: M128 N256"},
       {64, 16, 8, 1, 2, "uniform descs: M64 N16"},
       {128, 16, 8, 1, 3, "2 warps concurrently, M128 N16 (per MMA of all)"},
+      {128, 16, 8, 1, 4, "per-box C++ mbarrier poll + syncwarp, M128 N16"},
+      {128, 16, 8, 1, 5, "per-box PTX spin-loop wait, M128 N16"},
       {64, 16, 8, 1, 3, "2 warps concurrently, M64 N16 (per MMA of all)"},
   };
   for (auto& c : cfgs) {
