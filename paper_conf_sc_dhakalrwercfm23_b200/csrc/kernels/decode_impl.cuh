@@ -166,6 +166,7 @@ struct Smem {
   uint64_t* empty;           // [n_stages] MMA -> TMA
   uint64_t* tfull;           // [kAccSlots] MMA -> epilogue
   uint64_t* tempty;          // [kAccSlots] epilogue -> MMA
+  uint64_t* actbar;          // operand image bulk copy -> consumers
   unsigned long long* best;  // [8]
   int* tok;                  // [8]
   float* wsum;               // [kConsumerWarps][8]
@@ -196,6 +197,8 @@ __device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax, int 
   p += kAccSlots * 8;
   s.tempty = reinterpret_cast<uint64_t*>(p);
   p += kAccSlots * 8;
+  s.actbar = reinterpret_cast<uint64_t*>(p);
+  p += 8;
   s.best = reinterpret_cast<unsigned long long*>(p);
   p += 8 * 8;
   s.tok = reinterpret_cast<int*>(p);
@@ -232,14 +235,33 @@ __device__ __forceinline__ void split8(const float (&f)[8], uint4& hi, uint4& lo
                   l[4] | ((uint32_t)l[5] << 16), l[6] | ((uint32_t)l[7] << 16));
 }
 
-// One activation element (sequence b, segment column col) into the operand.
+// One activation element (sequence b, column col) into an operand laid out as
+// above: the shared-memory operand (segment column) or a global operand image
+// (input column).
 template <int B>
-__device__ __forceinline__ void act_store1(const Smem& sm, int b, int col, float v) {
+__device__ __forceinline__ void act_store1(uint8_t* base, int b, int col, float v) {
   const uint16_t h = f32_to_bf16_rne(v);
   const uint16_t l = f32_to_bf16_rne(v - bf16_bits_to_f32(h));
   const uint32_t e = (uint32_t)(col & 7) * 2u;
-  *reinterpret_cast<uint16_t*>(sm.act + act_off<B>(b, col >> 3) + e) = h;
-  *reinterpret_cast<uint16_t*>(sm.act + act_off<B>(decode_act_lo(B) + b, col >> 3) + e) = l;
+  *reinterpret_cast<uint16_t*>(base + act_off<B>(b, col >> 3) + e) = h;
+  *reinterpret_cast<uint16_t*>(base + act_off<B>(decode_act_lo(B) + b, col >> 3) + e) = l;
+}
+
+// Columns [n, round64(n)) of every sequence of an operand image: the last
+// block's padding, multiplied by weight columns past the input width (the
+// tensor maps read them from the next row). Written by the writer of column
+// n - 1: a slot's image is shared by tasks of different batch layouts.
+template <int B>
+__device__ __forceinline__ void img_zero_tail(uint8_t* img, int n) {
+  for (int c = n; c < round64(n); ++c)
+#pragma unroll
+    for (int b = 0; b < B; ++b) act_store1<B>(img, b, c, 0.f);
+}
+
+// Generic-proxy global writes (operand images) -> later async-proxy reads
+// (bulk copies issued by other CTAs after the grid barrier).
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
 // Device-wide barrier among all CTAs of the launch (consumer warps only; the
@@ -467,7 +489,7 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
     if (lane == 0) mbar_arrive(&sm.tempty[slot]);
     const int row = rt + 32 * q + lane;
     const bool ok = row < r1;
-    float v[B], u[B];
+    float v[B], u[B], xn[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       v[b] = __uint_as_float(d0[b]) + __uint_as_float(d0[LO + b]);
@@ -477,6 +499,7 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       key[b] = 0ull;
+      xn[b] = 0.f;
       if (!ok) continue;
       if (ph.nseg > 1) {
         float* acc = p.kacc + (size_t)b * ph.R * (gu ? 2 : 1);
@@ -491,16 +514,52 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
           continue;
         }
       }
+      // normed phases: the operand held x * gain, so the RMSNorm scale of
+      // sequence b multiplies the output column here
       switch (KIND) {
-        case PH_QKV: p.qkv[b * p.qkv_rows + row] = v[b]; break;
+        case PH_QKV: p.qkv[b * p.qkv_rows + row] = v[b] * sm.inv[b]; break;
         case PH_O:
-        case PH_DOWN: p.x[b * p.d + row] += v[b]; break;
-        case PH_GU: p.a[b * p.ff + row] = v[b] / (1.0f + expf(-v[b])) * u[b]; break;
-        case PH_LM:
-          key[b] = argmax_key(v[b], (uint32_t)row);
-          if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = v[b];
+        case PH_DOWN: {
+          const float t = p.x[b * p.d + row] + v[b];
+          p.x[b * p.d + row] = t;
+          xn[b] = t;
           break;
+        }
+        case PH_GU: {
+          const float g = v[b] * sm.inv[b], up = u[b] * sm.inv[b];
+          act_store1<B>(p.img_a, b, row, g / (1.0f + expf(-g)) * up);
+          if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_a, ph.R);
+          break;
+        }
+        case PH_LM: {
+          const float y = v[b] * sm.inv[b];
+          key[b] = argmax_key(y, (uint32_t)row);
+          if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = y;
+          break;
+        }
         default: break;
+      }
+    }
+    if ((KIND == PH_O || KIND == PH_DOWN) && last_seg) {
+      // the next normed phase's input: x * gain as an operand image, and the
+      // sums of squares of x over 8-row groups (fixed xor tree: independent of
+      // the grid); row groups never straddle CTAs (my_rows cuts at multiples of 8)
+      const uint16_t* gn =
+          (KIND == PH_O) ? p.w_layers + (uint64_t)ph.layer * p.layer_stride + p.off_gmlp
+          : (ph.layer + 1 < p.L) ? p.w_layers + (uint64_t)(ph.layer + 1) * p.layer_stride + p.off_gattn
+                                 : p.g_final;
+      const float gr = ok ? bf16_bits_to_f32(gn[row]) : 0.f;
+#pragma unroll
+      for (int b = 0; b < B; ++b) {
+        float t = xn[b] * xn[b];
+        t += __shfl_xor_sync(0xffffffffu, t, 1);
+        t += __shfl_xor_sync(0xffffffffu, t, 2);
+        t += __shfl_xor_sync(0xffffffffu, t, 4);
+        if (ok) {
+          if ((lane & 7) == 0) p.ssq[b * (p.d >> 3) + (row >> 3)] = t;
+          act_store1<B>(p.img_x, b, row, xn[b] * gr);
+          if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_x, ph.R);
+        }
       }
     }
     if (KIND == PH_LM && last_seg) {
@@ -516,6 +575,7 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
       }
     }
   }
+  if (KIND == PH_O || KIND == PH_DOWN || KIND == PH_GU) fence_proxy_async_global();
 }
 
 template <int B>
@@ -694,10 +754,8 @@ __device__ __forceinline__ void attend_hd(const DecodeParams& p, const Smem& sm,
   for (int d = 0; d < DPL; ++d) {
     const int dd = lane * DPL + d;
     const float o = acc[d] / l_run;
-    if (to_smem)
-      act_store1<B>(sm, b, h * HD + dd, o);
-    else
-      p.o[(size_t)b * p.q_dim + h * HD + dd] = o;
+    act_store1<B>(to_smem ? sm.act : p.img_o, b, h * HD + dd, o);
+    if (!to_smem && b == 0 && h * HD + dd == p.q_dim - 1) img_zero_tail<B>(p.img_o, p.q_dim);
   }
   __syncwarp();
 }
@@ -724,20 +782,46 @@ __device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer
     const int b = it / p.H, h = it - b * p.H;
     attend<B>(p, sm, layer, t, b, h, (h % group) == 0, false, warp, lane);
   }
+  // o image -> the O phase's bulk copies; the scratch (inside the operand
+  // region) -> the next bulk copy into it
+  fence_proxy_async_global();
+  fence_proxy_async();
 }
 
 // ---------------------------------------------------------------------------
-// Phase input -> activation operand (RMSNorm'd where the block says so). An
-// item is 8 consecutive columns of one sequence: two float4 loads (one uint4
-// of bf16 for the embedding rows), issued before any use so a segment costs one
-// L2 round trip when it fits kCache items per thread (the values then stay in
-// registers for the norm); wider inputs are read twice (norm, then staging).
+// Phase input -> activation operand. The phase that produces an input writes
+// it as a global operand image (act_store1 layout, x already multiplied by the
+// next norm's gain), so staging a K segment is ONE bulk copy of its blocks;
+// the RMSNorm scale 1/rms(x) of sequence b is a per-column factor of the
+// GEMV's output, applied by the epilogue (sm.inv), and rms(x) is reduced here
+// from the producer's 8-row sums of squares while the copy is in flight.
+// Exceptions: the layer-0 QKV input (embedding rows of the tokens, staged
+// item by item) and the fused-attention O input (computed into the operand).
 // ---------------------------------------------------------------------------
 constexpr int kCache = 2;
 
+// Fixed-order RMSNorm reduction of the per-thread partials acc[b]: warp
+// shuffle trees, then warps in order; sm.inv[b] = 1 / sqrt(mean + eps).
+template <int B>
+__device__ __forceinline__ void norm_finish(const DecodeParams& p, const Smem& sm, float (&acc)[B],
+                                            int KF, int tid_c) {
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+#pragma unroll
+  for (int b = 0; b < B; ++b) {
+    const float t = warp_sum(acc[b]);
+    if (lane == 0) sm.wsum[warp * 8 + b] = t;
+  }
+  named_bar_sync(1, kNCT);
+  if (tid_c < B) {
+    float t = 0.f;
+    for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + tid_c];
+    sm.inv[tid_c] = 1.0f / sqrtf(t / (float)KF + p.eps);
+  }
+}
+
 template <int B>
 __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm, const Phase& ph,
-                                          int s, int tid_c) {
+                                          int s, int tid_c, uint32_t& act_par) {
   const int kind = ph.kind, layer = ph.layer;
   const int cta = blockIdx.x, C = p.n_ctas;
   const int warp = tid_c >> 5, lane = tid_c & 31;
@@ -764,51 +848,67 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
     named_bar_sync(1, kNCT);
     return;
   }
-  const uint16_t* gain = nullptr;
-  const uint16_t* emb = nullptr;   // layer-0 input: the embedding rows of the tokens
-  const float* src = nullptr;
-  if (kind == PH_QKV && layer == 0) {
-    if (ph.seg == 0) {
-      // input token: prompt for s < P, else the argmax of step s-1 (reduced from
-      // the per-CTA candidates, identically in every CTA).
-      if (tid_c < B) {
-        int tok;
-        if (s < p.P) {
-          tok = p.prompt[tid_c * p.P + s];
-        } else {
-          unsigned long long best = 0;
-          for (int c = 0; c < C; ++c) {
-            const unsigned long long v = p.cand[c * B + tid_c];
-            best = v > best ? v : best;
-          }
-          tok = (int)argmax_key_index(best);
-          if (cta == 0) {
-            p.tokens[tid_c * p.G + (s - p.P)] = tok;
-            __threadfence_system();   // ordered before the completion flag
-          }
-        }
-        sm.tok[tid_c] = tok;
-      }
-      named_bar_sync(1, kNCT);
+  const bool normed = (kind == PH_QKV || kind == PH_GU || kind == PH_LM);
+  if (!(kind == PH_QKV && layer == 0)) {
+    // --- operand image: one bulk copy of the segment's blocks ---------------
+    if (tid_c == 0) {
+      const uint8_t* img = (kind == PH_O) ? p.img_o : (kind == PH_DOWN) ? p.img_a : p.img_x;
+      const uint32_t blk = (uint32_t)decode_act_blk_bytes(B);
+      const uint32_t bytes = (uint32_t)ph.nkb * blk;
+      const uint8_t* src = img + (size_t)(k0 / kBlkK) * blk;
+      fence_proxy_async_global();
+      mbar_arrive_expect_tx(sm.actbar, bytes);
+      for (uint32_t o = 0; o < bytes; o += 16384u)
+        bulk_g2s(sm.act + o, src + o, min(16384u, bytes - o), sm.actbar);
     }
-    emb = p.embed;
-    gain = p.w_layers + p.off_gattn;
-  } else {
-    src = (kind == PH_O) ? p.o : (kind == PH_DOWN) ? p.a : p.x;
-    if (kind == PH_QKV) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gattn;
-    if (kind == PH_GU) gain = p.w_layers + (uint64_t)layer * p.layer_stride + p.off_gmlp;
-    if (kind == PH_LM) gain = p.g_final;
+    if (normed && ph.seg == 0) {
+      // rms(x) from the producer's sums of squares over 8-row groups; the
+      // group -> thread assignment depends only on kNCT (not on the grid)
+      const int G8 = KF >> 3;
+      float acc[B];
+#pragma unroll
+      for (int b = 0; b < B; ++b) acc[b] = 0.f;
+      for (int g = tid_c; g < G8; g += kNCT) {
+#pragma unroll
+        for (int b = 0; b < B; ++b) acc[b] += p.ssq[b * G8 + g];
+      }
+      norm_finish<B>(p, sm, acc, KF, tid_c);
+    }
+    while (!mbar_try_wait(sm.actbar, act_par)) {
+    }
+    act_par ^= 1u;
+    named_bar_sync(1, kNCT);
+    return;
   }
+  // --- layer-0 QKV: embedding rows of the step's tokens ---------------------
+  if (ph.seg == 0) {
+    // input token: prompt for s < P, else the argmax of step s-1 (reduced from
+    // the per-CTA candidates, identically in every CTA).
+    if (tid_c < B) {
+      int tok;
+      if (s < p.P) {
+        tok = p.prompt[tid_c * p.P + s];
+      } else {
+        unsigned long long best = 0;
+        for (int c = 0; c < C; ++c) {
+          const unsigned long long v = p.cand[c * B + tid_c];
+          best = v > best ? v : best;
+        }
+        tok = (int)argmax_key_index(best);
+        if (cta == 0) {
+          p.tokens[tid_c * p.G + (s - p.P)] = tok;
+          __threadfence_system();   // ordered before the completion flag
+        }
+      }
+      sm.tok[tid_c] = tok;
+    }
+    named_bar_sync(1, kNCT);
+  }
+  const uint16_t* emb = p.embed;
+  const uint16_t* gain = p.w_layers + p.off_gattn;
   // 8 input values of sequence b at input column col (col < KF)
   auto load8 = [&](int b, int col, float (&f)[8]) {
-    if (emb) {
-      unpack8(*reinterpret_cast<const uint4*>(emb + (size_t)sm.tok[b] * KF + col), f);
-    } else {
-      const float4 a = *reinterpret_cast<const float4*>(src + (size_t)b * KF + col);
-      const float4 c = *reinterpret_cast<const float4*>(src + (size_t)b * KF + col + 4);
-      f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w;
-      f[4] = c.x; f[5] = c.y; f[6] = c.z; f[7] = c.w;
-    }
+    unpack8(*reinterpret_cast<const uint4*>(emb + (size_t)sm.tok[b] * KF + col), f);
   };
   const int n_items = B * nq;
   // single pass: the whole input is this segment and fits the register cache
@@ -827,10 +927,8 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
       }
     }
   }
-  if (gain && ph.seg == 0) {
-    // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt):
-    // per-thread partials, warp shuffle trees, fixed-order sum over warps; the
-    // scale is kept in smem for later K segments.
+  if (ph.seg == 0) {
+    // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt)
     float acc[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) acc[b] = 0.f;
@@ -869,35 +967,21 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
         }
       }
     }
-#pragma unroll
-    for (int b = 0; b < B; ++b) {
-      const float t = warp_sum(acc[b]);
-      if (lane == 0) sm.wsum[warp * 8 + b] = t;
-    }
-    named_bar_sync(1, kNCT);
-    if (tid_c < B) {
-      float t = 0.f;
-      for (int w = 0; w < kConsumerWarps; ++w) t += sm.wsum[w * 8 + tid_c];
-      sm.inv[tid_c] = 1.0f / sqrtf(t / (float)KF + p.eps);
-    }
-    named_bar_sync(1, kNCT);
+    norm_finish<B>(p, sm, acc, KF, tid_c);
   }
-  // scale (norm and gain), split hi/lo, store; columns >= K are zero
+  // x (CTA 0), gain-scaled operand split hi/lo; columns >= K are zero
   auto put = [&](int i, float (&f)[8]) {
     const int b = i / nq, q = i - b * nq;
     const int col = k0 + q * 8;
     if (q * 8 < K) {
-      if (emb && cta == 0) {
+      if (cta == 0) {
         *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col) = make_float4(f[0], f[1], f[2], f[3]);
         *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col + 4) = make_float4(f[4], f[5], f[6], f[7]);
       }
-      if (gain) {
-        const float ib = sm.inv[b];
-        float g[8];
-        unpack8(*reinterpret_cast<const uint4*>(gain + col), g);
+      float g[8];
+      unpack8(*reinterpret_cast<const uint4*>(gain + col), g);
 #pragma unroll
-        for (int j = 0; j < 8; ++j) f[j] = f[j] * ib * g[j];
-      }
+      for (int j = 0; j < 8; ++j) f[j] = f[j] * g[j];
     } else {
 #pragma unroll
       for (int j = 0; j < 8; ++j) f[j] = 0.f;
@@ -948,6 +1032,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
       mbar_init(&sm.tfull[i], 1);
       mbar_init(&sm.tempty[i], 4);
     }
+    mbar_init(sm.actbar, 1);
     fence_mbar_init();
     if (blockIdx.x == 0) p.stamps[0] = globaltimer();
   }
@@ -969,7 +1054,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
   const int tid_c = threadIdx.x - 32;
   const int L = p.L, S = p.P + p.G - 1;
   const int pl = phases_per_layer(p.fuse_att);
-  uint32_t stage = 0, phase_bit = 0, tc = 0;
+  uint32_t stage = 0, phase_bit = 0, tc = 0, act_par = 0;
   unsigned long long target = p.bar_base;
   long long c_bar = 0, c_stage = 0, c_gemv = 0, c_att = 0, w_full = 0, w_acc = 0, w_tf = 0;
   const long long t_begin = MX_CLK();
@@ -988,7 +1073,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         const int nseg = phase_segments<B>(p, kind);
         for (int seg = 0; seg < nseg; ++seg) {
           const Phase ph = make_phase<B>(p, kind, layer, seg);
-          stage_act<B>(p, sm, ph, s, tid_c);
+          stage_act<B>(p, sm, ph, s, tid_c, act_par);
           const long long t1 = MX_CLK();
           if (kind == PH_O && p.fuse_att)
             c_att += t1 - t0;

@@ -61,6 +61,13 @@ MX_HD constexpr int decode_act_bytes(int B, int kmax) {
           kBlkK) *
          decode_act_blk_bytes(B);
 }
+// Bytes of a global image of the activation operand over `cols` input columns
+// (the shared-memory layout above, every 64-column block): the phase that
+// produces an input writes it in this form, the consuming phase copies each
+// K segment into shared memory with one bulk copy.
+MX_HD constexpr int decode_img_bytes(int B, int cols) {
+  return ((cols + kBlkK - 1) / kBlkK) * decode_act_blk_bytes(B);
+}
 
 // One decode task on one partition: all P+G-1 steps in ONE persistent launch
 // (grid = the partition's SMs, one CTA per SM), phases separated by a
@@ -84,6 +91,12 @@ struct DecodeParams {
   float* qkv;                // [B][qkv_rows]
   float* o;                  // [B][q_dim]
   float* a;                  // [B][ff]
+  // operand images (decode_img_bytes): x * gain of the next normed phase (GU,
+  // QKV of the next layer, LM head), attention output o, MLP activation a
+  uint8_t* img_x;
+  uint8_t* img_o;
+  uint8_t* img_a;
+  float* ssq;                // [B][d / 8] sums of squares of x over 8-row groups
   unsigned long long* cand;  // [kMaxCtas][B] per-CTA argmax keys
   float* kacc;               // split-K partial sums [B][2 * max(qkv_rows, ff, d, V)]
   uint16_t* kc;              // [L][B][Hkv][max_seq][hd] bf16

@@ -492,6 +492,11 @@ static int alloc_decode_slot(Partition& p, FnInst& fi, Slot& s) {
   if ((rc = alloc_ptr(p, B * (q + 2 * kv) * 4, &s.qkv))) return rc;
   if ((rc = alloc_ptr(p, B * q * 4, &s.o))) return rc;
   if ((rc = alloc_ptr(p, B * ff * 4, &s.a))) return rc;
+  // operand images sized for the widest layout (16 operand rows, B > 4)
+  if ((rc = alloc_ptr(p, mxk::decode_img_bytes(8, (int)d), &s.img_x))) return rc;
+  if ((rc = alloc_ptr(p, mxk::decode_img_bytes(8, (int)q), &s.img_o))) return rc;
+  if ((rc = alloc_ptr(p, mxk::decode_img_bytes(8, (int)ff), &s.img_a))) return rc;
+  if ((rc = alloc_ptr(p, B * (d / 8) * 4, &s.ssq))) return rc;
   if ((rc = alloc_ptr(p, (uint64_t)mxk::kMaxCtas * B * 8, &s.cand))) return rc;
   const uint64_t kacc_rows = std::max(std::max(q + 2 * kv, 2 * ff), std::max(d, V));
   if ((rc = alloc_ptr(p, B * kacc_rows * 4, &s.kacc))) return rc;
@@ -766,6 +771,18 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
       set_error("slot reset failed");
       return fail(MX_EDEVICE);
     }
+    if (d.kind == MX_FN_DECODE) {
+      // operand images: columns past the input width and rows of absent
+      // sequences are never written by the kernel and must read as zero
+      const mx_decode_cfg& c = d.dec;
+      const int q = c.n_heads * c.head_dim;
+      if (drv().cuMemsetD8Async(s.img_x, 0, mxk::decode_img_bytes(8, c.d_model), st) != CUDA_SUCCESS ||
+          drv().cuMemsetD8Async(s.img_o, 0, mxk::decode_img_bytes(8, q), st) != CUDA_SUCCESS ||
+          drv().cuMemsetD8Async(s.img_a, 0, mxk::decode_img_bytes(8, c.d_ff), st) != CUDA_SUCCESS) {
+        set_error("slot reset failed");
+        return fail(MX_EDEVICE);
+      }
+    }
   }
   if (drv().cuStreamSynchronize(st) != CUDA_SUCCESS) {
     set_error("cold start on partition %d failed on the device", p.id);
@@ -877,6 +894,10 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.qkv = reinterpret_cast<float*>(s.qkv);
     k.o = reinterpret_cast<float*>(s.o);
     k.a = reinterpret_cast<float*>(s.a);
+    k.img_x = reinterpret_cast<uint8_t*>(s.img_x);
+    k.img_o = reinterpret_cast<uint8_t*>(s.img_o);
+    k.img_a = reinterpret_cast<uint8_t*>(s.img_a);
+    k.ssq = reinterpret_cast<float*>(s.ssq);
     k.cand = reinterpret_cast<unsigned long long*>(s.cand);
     k.kacc = reinterpret_cast<float*>(s.kacc);
     k.kc = reinterpret_cast<uint16_t*>(s.kc);
