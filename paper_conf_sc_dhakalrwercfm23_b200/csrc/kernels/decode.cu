@@ -18,7 +18,7 @@ int decode_smem_bytes(int B, int kmax, int* n_stages, int fuse_att) {
   // mbarriers (TMEM slots, operand copy) + small scratch; the rest is the weight ring
   const int att = decode_att_in_act(B, kmax, fuse_att) ? 0 : kConsumerWarps * 3 * kAttHd * 4;
   const int fixed = 1024 + decode_act_bytes(B, kmax) + att +
-                    4 * 2 * 8 + 8 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 16;
+                    4 * 2 * 8 + 32 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 16;
   const int per_stage = kStageBytes + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;

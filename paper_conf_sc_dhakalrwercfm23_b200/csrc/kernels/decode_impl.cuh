@@ -51,9 +51,10 @@ enum DecodeMat { MAT_QKV = 0, MAT_O = 1, MAT_GATE = 2, MAT_UP = 3, MAT_DOWN = 4,
 constexpr int kNCT = 32 * kConsumerWarps;   // consumer threads
 constexpr int kMmaWarp = 1;                 // warp whose lane 0 issues the MMAs
 constexpr int kEpiWarp0 = 2;                // warps 2..5 drain TMEM (lane quarter = warp % 4)
+constexpr int kStageWarp = 6;               // lane 0 copies the operand images (bulk copies)
 constexpr int kAccSlots = 4;                // TMEM accumulator slots of 32 columns
 #ifndef MX_MMA_WARP
-#define MX_MMA_WARP 1                       // 1: warp-uniform issue, elected lane (see tc05.cuh)
+#define MX_MMA_WARP 2                       // 1: warp-wide issue, one elect per MMA; 2: one elect per K block (tc05.cuh)
 #endif
 constexpr uint32_t kTmemCols = 32 * kAccSlots;
 static_assert(kConsumerWarps >= 5, "MMA warp + 4 epilogue warps");
@@ -107,6 +108,19 @@ struct Phase {
 
 __host__ __device__ __forceinline__ int round64(int k) { return (k + 63) & ~63; }
 
+// K segments of a phase: one when the input fits the operand region (64 KiB),
+// else segments of at most half of it, so that the operand of segment s + 1 is
+// copied into one half while the MMAs of segment s read the other.
+template <int B>
+__device__ __forceinline__ int phase_segments(const DecodeParams& p, int kind) {
+  if (kind == PH_ATT) return 1;
+  const int KF = (kind == PH_O) ? p.q_dim : (kind == PH_DOWN) ? p.ff : p.d;
+  constexpr int SEG = decode_seg_cols(B);
+  if (KF <= SEG) return 1;
+  constexpr int SEG2 = SEG / 2;
+  return (KF + SEG2 - 1) / SEG2;
+}
+
 template <int B>
 __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int layer, int seg) {
   Phase ph;
@@ -120,8 +134,7 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
     case PH_DOWN: ph.R = p.d; ph.KF = p.ff; ph.mat = MAT_DOWN; break;
     default: ph.R = p.V; ph.KF = p.d; ph.mat = MAT_LM; ph.lz = 0; break;
   }
-  constexpr int SEG = decode_seg_cols(B);
-  ph.nseg = max(1, (ph.KF + SEG - 1) / SEG);
+  ph.nseg = phase_segments<B>(p, kind);
   const int w = (ph.nseg == 1) ? round64(ph.KF)
                                : ((ph.KF + ph.nseg - 1) / ph.nseg + kSegGrain - 1) / kSegGrain * kSegGrain;
   ph.seg = seg;
@@ -131,13 +144,6 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
   return ph;
 }
 
-template <int B>
-__device__ __forceinline__ int phase_segments(const DecodeParams& p, int kind) {
-  if (kind == PH_ATT) return 1;
-  const int KF = (kind == PH_O) ? p.q_dim : (kind == PH_DOWN) ? p.ff : p.d;
-  constexpr int SEG = decode_seg_cols(B);
-  return max(1, (KF + SEG - 1) / SEG);
-}
 
 // Rows [r0, r1) of a phase owned by this CTA: boundaries at multiples of 8
 // (the last is R); `rot` rotates the assignment so remainders land on
@@ -166,7 +172,8 @@ struct Smem {
   uint64_t* empty;           // [n_stages] MMA -> TMA
   uint64_t* tfull;           // [kAccSlots] MMA -> epilogue
   uint64_t* tempty;          // [kAccSlots] epilogue -> MMA
-  uint64_t* actbar;          // operand image bulk copy -> consumers
+  uint64_t* actfull;         // [2] operand half: bulk copy -> MMA
+  uint64_t* actfree;         // [2] operand half: MMAs done -> next bulk copy
   unsigned long long* best;  // [8]
   int* tok;                  // [8]
   float* wsum;               // [kConsumerWarps][8]
@@ -197,8 +204,10 @@ __device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax, int 
   p += kAccSlots * 8;
   s.tempty = reinterpret_cast<uint64_t*>(p);
   p += kAccSlots * 8;
-  s.actbar = reinterpret_cast<uint64_t*>(p);
-  p += 8;
+  s.actfull = reinterpret_cast<uint64_t*>(p);
+  p += 16;
+  s.actfree = reinterpret_cast<uint64_t*>(p);
+  p += 16;
   s.best = reinterpret_cast<unsigned long long*>(p);
   p += 8 * 8;
   s.tok = reinterpret_cast<int*>(p);
@@ -383,10 +392,11 @@ template <int B>
 __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                           int k, uint32_t& stage, uint32_t& phase_bit,
                                           int n_stages, uint32_t& tc, uint32_t tmem_base,
-                                          long long& w_full, long long& w_acc) {
+                                          long long& w_full, long long& w_acc,
+                                          uint32_t act_byte_off = 0) {
   constexpr uint32_t idesc = umma_idesc_bf16(kTileM, 16);
   constexpr uint32_t sbo = (B <= 4) ? 0u : 1024u;   // B <= 4: the 8-row atom is read twice
-  const uint32_t act0 = smem_u32(sm.act), ring0 = smem_u32(sm.ring);
+  const uint32_t act0 = smem_u32(sm.act) + act_byte_off, ring0 = smem_u32(sm.ring);
   const int nm = (ph.kind == PH_GU) ? 2 : 1;
   const bool lane0 = (threadIdx.x & 31) == 0;
   (void)lane0;
@@ -418,7 +428,9 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
           const uint64_t ad = umma_desc_sw128(sa + (uint32_t)(j * h8 * 128));
           const uint64_t bd =
               umma_desc_sw128(act0 + (uint32_t)((kb + j) * decode_act_blk_bytes(B)), sbo);
-#if MX_MMA_WARP
+#if MX_MMA_WARP == 2
+          umma_f16_warp_k64(d, ad, bd, idesc, (kb + j > 0) ? 1u : 0u);
+#elif MX_MMA_WARP
 #pragma unroll
           for (int jj = 0; jj < kBlkK / 16; ++jj)
             umma_f16_warp(d, ad + 2u * (uint32_t)jj, bd + 2u * (uint32_t)jj, idesc,
@@ -819,9 +831,55 @@ __device__ __forceinline__ void norm_finish(const DecodeParams& p, const Smem& s
   }
 }
 
+// Operand-image phases, all consumer threads: reset the LM argmax, reduce
+// rms(x) from the producer's sums of squares over 8-row groups (the group ->
+// thread assignment depends only on kNCT, not on the grid).
+template <int B>
+__device__ __forceinline__ void prep_img(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                         int tid_c) {
+  if (ph.kind == PH_LM && tid_c < B) sm.best[tid_c] = 0ull;
+  if (ph.kind == PH_QKV || ph.kind == PH_GU || ph.kind == PH_LM) {
+    const int G8 = ph.KF >> 3;
+    float acc[B];
+#pragma unroll
+    for (int b = 0; b < B; ++b) acc[b] = 0.f;
+    for (int g = tid_c; g < G8; g += kNCT) {
+#pragma unroll
+      for (int b = 0; b < B; ++b) acc[b] += p.ssq[b * G8 + g];
+    }
+    norm_finish<B>(p, sm, acc, ph.KF, tid_c);
+  }
+  named_bar_sync(1, kNCT);
+}
+
+__device__ __forceinline__ bool img_phase(const DecodeParams& p, int kind, int layer) {
+  return !(kind == PH_QKV && layer == 0) && !(kind == PH_O && p.fuse_att);
+}
+
+// Operand-image phases, one thread: copy segment ph's blocks of the image into
+// operand half `buf` (the whole region when the phase has one segment) once the
+// MMAs of that half's previous use (`use` - 1) have completed.
+template <int B>
+__device__ __forceinline__ void issue_img_copy(const DecodeParams& p, const Smem& sm,
+                                               const Phase& ph, uint32_t buf, uint32_t use) {
+  if (use > 0) {
+    while (!mbar_try_wait(&sm.actfree[buf], (use - 1) & 1u)) {
+    }
+  }
+  const uint8_t* img = (ph.kind == PH_O) ? p.img_o : (ph.kind == PH_DOWN) ? p.img_a : p.img_x;
+  const uint32_t blk = (uint32_t)decode_act_blk_bytes(B);
+  const uint32_t bytes = (uint32_t)ph.nkb * blk;
+  const uint8_t* src = img + (size_t)(ph.k0 / kBlkK) * blk;
+  uint8_t* dst = sm.act + buf * (uint32_t)(decode_act_bytes(B, decode_seg_cols(B)) / 2);
+  fence_proxy_async_global();
+  mbar_arrive_expect_tx(&sm.actfull[buf], bytes);
+  for (uint32_t o = 0; o < bytes; o += 16384u)
+    bulk_g2s(dst + o, src + o, min(16384u, bytes - o), &sm.actfull[buf]);
+}
+
 template <int B>
 __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm, const Phase& ph,
-                                          int s, int tid_c, uint32_t& act_par) {
+                                          int s, int tid_c) {
   const int kind = ph.kind, layer = ph.layer;
   const int cta = blockIdx.x, C = p.n_ctas;
   const int warp = tid_c >> 5, lane = tid_c & 31;
@@ -845,38 +903,6 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
       attend<B>(p, sm, layer, s, b, h, cta == 0 && (h % group) == 0, true, warp, lane);
     }
     fence_proxy_async();
-    named_bar_sync(1, kNCT);
-    return;
-  }
-  const bool normed = (kind == PH_QKV || kind == PH_GU || kind == PH_LM);
-  if (!(kind == PH_QKV && layer == 0)) {
-    // --- operand image: one bulk copy of the segment's blocks ---------------
-    if (tid_c == 0) {
-      const uint8_t* img = (kind == PH_O) ? p.img_o : (kind == PH_DOWN) ? p.img_a : p.img_x;
-      const uint32_t blk = (uint32_t)decode_act_blk_bytes(B);
-      const uint32_t bytes = (uint32_t)ph.nkb * blk;
-      const uint8_t* src = img + (size_t)(k0 / kBlkK) * blk;
-      fence_proxy_async_global();
-      mbar_arrive_expect_tx(sm.actbar, bytes);
-      for (uint32_t o = 0; o < bytes; o += 16384u)
-        bulk_g2s(sm.act + o, src + o, min(16384u, bytes - o), sm.actbar);
-    }
-    if (normed && ph.seg == 0) {
-      // rms(x) from the producer's sums of squares over 8-row groups; the
-      // group -> thread assignment depends only on kNCT (not on the grid)
-      const int G8 = KF >> 3;
-      float acc[B];
-#pragma unroll
-      for (int b = 0; b < B; ++b) acc[b] = 0.f;
-      for (int g = tid_c; g < G8; g += kNCT) {
-#pragma unroll
-        for (int b = 0; b < B; ++b) acc[b] += p.ssq[b * G8 + g];
-      }
-      norm_finish<B>(p, sm, acc, KF, tid_c);
-    }
-    while (!mbar_try_wait(sm.actbar, act_par)) {
-    }
-    act_par ^= 1u;
     named_bar_sync(1, kNCT);
     return;
   }
@@ -1022,7 +1048,9 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
                                                                    int kmax) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   const Smem sm = carve<B>(smem_raw, n_stages, kmax, p.fuse_att);
-  const int warp_id = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // warp index through a shuffle: provably warp-uniform, so role branches are
+  // uniform and the MMA descriptors stay in uniform registers
+  const int warp_id = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int i = 0; i < n_stages; ++i) {
       mbar_init(&sm.full[i], 1);
@@ -1032,7 +1060,10 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
       mbar_init(&sm.tfull[i], 1);
       mbar_init(&sm.tempty[i], 4);
     }
-    mbar_init(sm.actbar, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&sm.actfull[i], 1);
+      mbar_init(&sm.actfree[i], 1);
+    }
     fence_mbar_init();
     if (blockIdx.x == 0) p.stamps[0] = globaltimer();
   }
@@ -1054,9 +1085,10 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
   const int tid_c = threadIdx.x - 32;
   const int L = p.L, S = p.P + p.G - 1;
   const int pl = phases_per_layer(p.fuse_att);
-  uint32_t stage = 0, phase_bit = 0, tc = 0, act_par = 0;
+  uint32_t stage = 0, phase_bit = 0, tc = 0;
+  uint32_t img_seq = 0, act_use[2] = {0u, 0u}, mma_use[2] = {0u, 0u};
   unsigned long long target = p.bar_base;
-  long long c_bar = 0, c_stage = 0, c_gemv = 0, c_att = 0, w_full = 0, w_acc = 0, w_tf = 0;
+  long long c_bar = 0, c_stage = 0, c_gemv = 0, c_att = 0, w_full = 0, w_acc = 0, w_tf = 0, w_act = 0;
   const long long t_begin = MX_CLK();
   for (int s = 0; s < S; ++s) {
     const int nph = pl * L + (s >= p.P - 1 ? 1 : 0);
@@ -1071,22 +1103,65 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         t0 = t1;
       } else {
         const int nseg = phase_segments<B>(p, kind);
-        for (int seg = 0; seg < nseg; ++seg) {
-          const Phase ph = make_phase<B>(p, kind, layer, seg);
-          stage_act<B>(p, sm, ph, s, tid_c, act_par);
+        if (img_phase(p, kind, layer)) {
+          // segment s + 1's operand is copied into one half while the MMAs of
+          // segment s read the other (kStageWarp lane 0 runs the copies)
+          const uint32_t img0 = img_seq;
+          img_seq += (uint32_t)nseg;
+          const bool stager = (warp_id == kStageWarp);   // lane 0 issues, the warp stays converged
+          auto half = [&](int seg) { return nseg == 1 ? 0u : (img0 + (uint32_t)seg) & 1u; };
+          auto copy_seg = [&](int seg) {
+            const uint32_t hb = half(seg);
+            if (lane == 0) issue_img_copy<B>(p, sm, make_phase<B>(p, kind, layer, seg), hb, act_use[hb]);
+            ++act_use[hb];
+            __syncwarp();
+          };
+          if (stager) copy_seg(0);
+          prep_img<B>(p, sm, make_phase<B>(p, kind, layer, 0), tid_c);
           const long long t1 = MX_CLK();
-          if (kind == PH_O && p.fuse_att)
-            c_att += t1 - t0;
-          else
-            c_stage += t1 - t0;
-          if (warp_id == kMmaWarp) {
-            mma_phase<B>(p, sm, ph, k, stage, phase_bit, n_stages, tc, tmem_base, w_full, w_acc);
+          c_stage += t1 - t0;
+          if (stager) {
+            for (int seg = 1; seg < nseg; ++seg) copy_seg(seg);
+          } else if (warp_id == kMmaWarp) {
+            for (int seg = 0; seg < nseg; ++seg) {
+              const Phase ph = make_phase<B>(p, kind, layer, seg);
+              const uint32_t hb = half(seg);
+              const long long tw = MX_CLK();
+              while (!mbar_try_wait(&sm.actfull[hb], mma_use[hb] & 1u)) {
+              }
+              __syncwarp();
+              w_act += MX_CLK() - tw;
+              ++mma_use[hb];
+              mma_phase<B>(p, sm, ph, k, stage, phase_bit, n_stages, tc, tmem_base, w_full, w_acc,
+                           hb * (uint32_t)(decode_act_bytes(B, decode_seg_cols(B)) / 2));
+              umma_commit_warp(smem_u32(&sm.actfree[hb]));   // half free once these MMAs completed
+            }
           } else if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
-            epi_dispatch<B>(p, sm, ph, k, s, warp_id, lane, tc, tmem_base, w_tf);
+            for (int seg = 0; seg < nseg; ++seg)
+              epi_dispatch<B>(p, sm, make_phase<B>(p, kind, layer, seg), k, s, warp_id, lane, tc,
+                              tmem_base, w_tf);
           }
           const long long t2 = MX_CLK();
           c_gemv += t2 - t1;
           t0 = t2;
+        } else {
+          for (int seg = 0; seg < nseg; ++seg) {
+            const Phase ph = make_phase<B>(p, kind, layer, seg);
+            stage_act<B>(p, sm, ph, s, tid_c);
+            const long long t1 = MX_CLK();
+            if (kind == PH_O && p.fuse_att)
+              c_att += t1 - t0;
+            else
+              c_stage += t1 - t0;
+            if (warp_id == kMmaWarp) {
+              mma_phase<B>(p, sm, ph, k, stage, phase_bit, n_stages, tc, tmem_base, w_full, w_acc);
+            } else if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
+              epi_dispatch<B>(p, sm, ph, k, s, warp_id, lane, tc, tmem_base, w_tf);
+            }
+            const long long t2 = MX_CLK();
+            c_gemv += t2 - t1;
+            t0 = t2;
+          }
         }
         if (kind == PH_LM) {
           named_bar_sync(1, kNCT);
@@ -1109,6 +1184,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     pr[7] = (unsigned long long)w_acc;
   }
   if (p.prof && tid_c == 32) p.prof[blockIdx.x * 16 + 8] = (unsigned long long)w_tf;
+  if (p.prof && tid_c == 0) p.prof[blockIdx.x * 16 + 9] = (unsigned long long)w_act;
   // final token (argmax of the last step)
   if (blockIdx.x == 0) {
     if (tid_c < B) {

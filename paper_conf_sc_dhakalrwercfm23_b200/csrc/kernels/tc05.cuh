@@ -65,6 +65,27 @@ __device__ __forceinline__ void umma_f16_warp(uint32_t tmem_d, uint64_t adesc, u
       : "memory");
 }
 
+// Warp-wide issue of the 4 MMAs of one 64-column K block (K = 16 each: the
+// descriptors advance by 32 bytes = 2 in the start-address field) under ONE
+// elect: the per-MMA operand moves to uniform registers are independent and
+// overlap instead of forming one elect -> move -> MMA chain per MMA.
+__device__ __forceinline__ void umma_f16_warp_k64(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc,
+                                                  uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred e, p, t;\n\t.reg .b64 a1, a2, a3, b1, b2, b3;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "setp.eq.u32 t, 0, 0;\n\t"
+      "add.s64 a1, %1, 2;\n\tadd.s64 a2, %1, 4;\n\tadd.s64 a3, %1, 6;\n\t"
+      "add.s64 b1, %2, 2;\n\tadd.s64 b2, %2, 4;\n\tadd.s64 b3, %2, 6;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], a1, b1, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], a2, b2, %3, t;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], a3, b3, %3, t;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
 __device__ __forceinline__ void umma_commit_warp(uint32_t bar_saddr) {
   asm volatile(
       "{\n\t.reg .pred e;\n\t"

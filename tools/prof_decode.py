@@ -51,7 +51,8 @@ if os.environ.get("MX_DECODE_PROF") == "1":
     n = mx.part_query(p)["n_ctas"]
     pr = mx.decode_profile(p, 2 * n).astype(float).reshape(n, 16)
     names = {0: "total", 1: "grid_barrier", 2: "stage_input", 3: "mma_wait_full", 4: "gemv(mma+epi)",
-             5: "attention", 6: "producer_wait", 7: "mma_wait_acc", 8: "epi_wait_tfull"}
+             5: "attention", 6: "producer_wait", 7: "mma_wait_acc", 8: "epi_wait_tfull",
+             9: "mma_wait_operand"}
     tot = pr[:, 0].mean()
     for i, nm in names.items():
         print(f"  {nm:16s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
