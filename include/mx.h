@@ -70,7 +70,7 @@ enum { MX_INIT_DEFAULT = 0 };
  * P:113-115 §3.2, §3.4, Fig. 4; block conventions C2/A8).
  * Constraints: d_model, q_dim = n_heads*head_dim and d_ff multiples of 8;
  * head_dim in {32, 64, 128}; n_heads % n_kv_heads == 0; 1 <= max_batch <= 8;
- * d_model <= 8192, q_dim and d_ff <= 16384. GEMVs run on the tensor cores
+ * d_model <= 8192, q_dim and d_ff <= 16384, vocab <= 2^20. GEMVs run on the tensor cores
  * (tcgen05); phases whose input is wider than 64 KiB of bf16 hi/lo operand
  * (4096 columns at batch <= 4, 2048 above) run as K segments (split-K).    */
 typedef struct {

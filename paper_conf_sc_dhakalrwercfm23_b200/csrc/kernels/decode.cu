@@ -18,7 +18,7 @@ int decode_smem_bytes(int B, int kmax, int* n_stages, int fuse_att) {
   // mbarriers (TMEM slots, operand copy) + small scratch; the rest is the weight ring
   const int att = decode_att_in_act(B, kmax, fuse_att) ? 0 : kConsumerWarps * 3 * kAttHd * 4;
   const int fixed = 1024 + decode_act_bytes(B, kmax) + att +
-                    4 * 2 * 8 + 32 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 16;
+                    4 * 2 * 8 + 32 + 8 * 8 + 8 * 4 + kConsumerWarps * 8 * 4 + 8 * 4 + 6 * 4 * 4 + 16;
   const int per_stage = kStageBytes + 16;
   const int cap = 227 * 1024;
   int ns = (cap - fixed) / per_stage;
@@ -42,6 +42,18 @@ int decode_prof_buckets() {
 // Fused attention (every CTA computes all heads inside the O phase) saves a
 // grid barrier per layer but replicates the K/V reads over the grid: used for
 // small attention on grids of at most MX_FUSE_MAX_CTAS CTAs.
+uint64_t decode_kpart_floats(int B, int d, int q_dim, int qkv_rows, int ff, int V, int fuse_att) {
+  // (rows, input width, gate/up pair, splittable) of QKV, O, GU, DOWN, LM
+  const long long sh[5][4] = {{qkv_rows, d, 1, 1}, {d, q_dim, 1, !fuse_att}, {ff, d, 2, 1},
+                              {d, ff, 1, 1}, {V, d, 1, 1}};
+  uint64_t m = 0;
+  for (const auto& t : sh) {
+    const int ns = decode_nseg(B, t[0], (int)t[1], (int)t[3]);
+    if (ns > 1) m = std::max(m, (uint64_t)ns * (uint64_t)t[0] * (uint64_t)t[2] * (uint64_t)B);
+  }
+  return m;
+}
+
 int decode_fuse_attention(int B, int H, int hd, int n_ctas) {
   return (B * H * hd <= 1024 && n_ctas <= MX_FUSE_MAX_CTAS) ? 1 : 0;
 }

@@ -104,6 +104,8 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
 // widths are multiples of 64 and depend only on the shape).
 struct Phase {
   int kind, layer, R, KF, K, k0, seg, nseg, nkb, mat, lz;
+  int w;     // full segment width (the last segment may be narrower: K)
+  int dist;  // multi-segment phase whose (segment, rows) pieces are spread over the CTAs
 };
 
 __host__ __device__ __forceinline__ int round64(int k) { return (k + 63) & ~63; }
@@ -115,10 +117,8 @@ template <int B>
 __device__ __forceinline__ int phase_segments(const DecodeParams& p, int kind) {
   if (kind == PH_ATT) return 1;
   const int KF = (kind == PH_O) ? p.q_dim : (kind == PH_DOWN) ? p.ff : p.d;
-  constexpr int SEG = decode_seg_cols(B);
-  if (KF <= SEG) return 1;
-  constexpr int SEG2 = SEG / 2;
-  return (KF + SEG2 - 1) / SEG2;
+  const int R = (kind == PH_QKV) ? p.qkv_rows : (kind == PH_GU) ? p.ff : (kind == PH_LM) ? p.V : p.d;
+  return decode_nseg(B, R, KF, !(kind == PH_O && p.fuse_att));
 }
 
 template <int B>
@@ -138,6 +138,12 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
   const int w = (ph.nseg == 1) ? round64(ph.KF)
                                : ((ph.KF + ph.nseg - 1) / ph.nseg + kSegGrain - 1) / kSegGrain * kSegGrain;
   ph.seg = seg;
+  ph.w = w;
+  // a plain row split would leave a CTA < 64 rows per MMA (issue-bound: a
+  // skinny MMA costs the same for 8 or 128 rows), so spread the pieces; else
+  // each CTA runs every segment of its rows and chains the partials itself.
+  // Either way the row's sum is ((p0 + p1) + p2) + ...: the same bits.
+  ph.dist = ((kind == PH_O || kind == PH_DOWN) && ph.nseg > 1 && ph.R < 64 * p.n_ctas) ? 1 : 0;
   ph.k0 = seg * w;
   ph.K = min(w, ph.KF - ph.k0);
   ph.nkb = (ph.K + kBlkK - 1) / kBlkK;
@@ -149,9 +155,68 @@ __device__ __forceinline__ Phase make_phase(const DecodeParams& p, int kind, int
 // (the last is R); `rot` rotates the assignment so remainders land on
 // different CTAs in different phases.
 __device__ __forceinline__ void my_rows(int R, int C, int cta, int rot, int* r0, int* r1) {
-  const int c = (cta + rot) % C;
-  *r0 = (int)(((long long)R * c) / C) & ~7;
-  *r1 = (c + 1 == C) ? R : ((int)(((long long)R * (c + 1)) / C) & ~7);
+  // 32-bit arithmetic: R * C < 2^32 for every admitted shape (R <= 2^24, C <= kMaxCtas)
+  const uint32_t c = (uint32_t)(cta + rot) % (uint32_t)C;
+  *r0 = (int)(((uint32_t)R * c) / (uint32_t)C) & ~7;
+  *r1 = (c + 1 == (uint32_t)C) ? R : ((int)(((uint32_t)R * (c + 1)) / (uint32_t)C) & ~7);
+}
+
+// Multi-segment phases: the work (segment g, 8-row group i), ordered segment-
+// major and weighted by the segment's width, is cut into n_ctas equal
+// contiguous ranges; CTA c's piece of segment g is the rows [r0, r1) of its
+// range inside g (empty for most g). Which CTA computes a partial does not
+// change its value, so results do not depend on the partition size.
+__device__ __forceinline__ void seg_pos(long long T, int G8, int w, int KF, int nseg, int* g,
+                                        int* i) {
+  const long long segW = (long long)G8 * w;
+  const int gg = (int)min(T / segW, (long long)(nseg - 1));
+  const int wg = min(w, KF - gg * w);
+  *g = gg;
+  *i = (int)min((T - gg * segW) / wg, (long long)G8);
+}
+
+// This CTA's pieces of a multi-segment phase kind (computed once per launch,
+// kept in shared memory): segments [ga, gb], rows [r0a, R) of ga ... rows
+// [0, r1b) of gb (ga > gb: none).
+__device__ __forceinline__ void cta_span(const Phase& ph, int C, int cta, int* sp) {
+  const int G8 = (ph.R + 7) >> 3;
+  const long long W = (long long)G8 * ph.KF;
+  int gs, is, ge, ie;
+  seg_pos(W * cta / C, G8, ph.w, ph.KF, ph.nseg, &gs, &is);
+  seg_pos(W * (cta + 1) / C, G8, ph.w, ph.KF, ph.nseg, &ge, &ie);
+  int ga = gs, r0a = is * 8, gb = ge, r1b = min(ie * 8, ph.R);
+  if (r0a >= ph.R) {
+    ++ga;
+    r0a = 0;
+  }
+  if (r1b <= 0) {
+    --gb;
+    r1b = ph.R;
+  }
+  if (ga > gb || (ga == gb && r0a >= r1b)) {
+    ga = 1;
+    gb = 0;
+  }
+  sp[0] = ga;
+  sp[1] = r0a;
+  sp[2] = gb;
+  sp[3] = r1b;
+}
+
+__device__ __forceinline__ void piece_rows(const Phase& ph, const int* span, int C, int cta, int k,
+                                           int* r0, int* r1) {
+  if (!ph.dist) {
+    my_rows(ph.R, C, cta, k, r0, r1);
+    return;
+  }
+  const int* sp = span + 4 * ph.kind;
+  const int g = ph.seg;
+  if (g < sp[0] || g > sp[2]) {
+    *r0 = *r1 = 0;
+    return;
+  }
+  *r0 = (g == sp[0]) ? sp[1] : 0;
+  *r1 = (g == sp[2]) ? sp[3] : ph.R;
 }
 
 __host__ __device__ __forceinline__ int phases_per_layer(int fuse_att) { return fuse_att ? 4 : 5; }
@@ -178,6 +243,7 @@ struct Smem {
   int* tok;                  // [8]
   float* wsum;               // [kConsumerWarps][8]
   float* inv;                // [8] RMSNorm scale of the phase input (kept across K segments)
+  int* span;                 // [6][4] this CTA's pieces per multi-segment phase kind (cta_span)
   uint32_t* tmem;            // TMEM base address
 };
 
@@ -216,6 +282,8 @@ __device__ __forceinline__ Smem carve(uint8_t* raw, int n_stages, int kmax, int 
   p += (size_t)kConsumerWarps * 8 * 4;
   s.inv = reinterpret_cast<float*>(p);
   p += 8 * 4;
+  s.span = reinterpret_cast<int*>(p);
+  p += 6 * 4 * 4;
   s.tmem = reinterpret_cast<uint32_t*>(p);
   return s;
 }
@@ -277,9 +345,10 @@ __device__ __forceinline__ void fence_proxy_async_global() {
 // producer warp never waits on it). A 4 s timeout sets *err; afterwards every
 // barrier passes without waiting, so a failed launch still terminates.
 __device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned long long target,
-                                             int tid_c) {
+                                             int tid_c, unsigned long long* tl = nullptr) {
   named_bar_sync(1, kNCT);
   if (tid_c == 0) {
+    if (tl) tl[4] = globaltimer();
     // release: this CTA's phase outputs (ordered before by bar.sync) become visible
     asm volatile("red.release.gpu.global.add.u64 [%0], 1;" ::"l"(p.bar) : "memory");
     if (!ld_volatile_i32(p.err)) {
@@ -298,6 +367,7 @@ __device__ __forceinline__ void grid_barrier(const DecodeParams& p, unsigned lon
     // acquire: one acquire load of the final count synchronizes with every CTA's
     // release RMW (and invalidates this SM's L1 once for the whole CTA)
     (void)ld_acquire_u64(p.bar);
+    if (tl) tl[5] = globaltimer();
   }
   named_bar_sync(1, kNCT);
 }
@@ -355,7 +425,7 @@ __device__ void producer_loop(const DecodeParams& p, const Smem& sm, int n_stage
         const Phase ph = make_phase<B>(p, kind, k / pl, seg);
         const int nm = (kind == PH_GU) ? 2 : 1;
         int r0, r1;
-        my_rows(ph.R, C, cta, k, &r0, &r1);
+        piece_rows(ph, sm.span, C, cta, k, &r0, &r1);
         for (int rt = r0; rt < r1; rt += kTileM) {
           const int h8 = (min(kTileM, r1 - rt) + 7) & ~7;
           const int nk = decode_box_blocks(h8);
@@ -401,7 +471,7 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
   const bool lane0 = (threadIdx.x & 31) == 0;
   (void)lane0;
   int r0, r1;
-  my_rows(ph.R, p.n_ctas, blockIdx.x, k, &r0, &r1);
+  piece_rows(ph, sm.span, p.n_ctas, blockIdx.x, k, &r0, &r1);
   for (int rt = r0; rt < r1; rt += kTileM) {
     const uint32_t slot = tc % kAccSlots, use = tc / kAccSlots;
     const long long ta = MX_CLK();
@@ -470,9 +540,93 @@ __device__ __forceinline__ void mma_phase(const DecodeParams& p, const Smem& sm,
 // ---------------------------------------------------------------------------
 // Epilogue warps: warp w reads TMEM lanes 32(w%4).. (tile rows) of each tile's
 // slot; column n of the accumulator is operand row n: sequence b's value is
-// D[b] + D[lo + b] (hi + lo parts). Split-K partials go through the slot's
-// kacc buffer (rows are owned by this CTA: no atomics).
+// D[b] + D[lo + b] (hi + lo parts). Single-segment phases finish each row
+// straight from TMEM; multi-segment phases store the segment's partial
+// (kpart) and the CTA completing a row block finishes it (epi_finalize).
 // ---------------------------------------------------------------------------
+
+// The phase's output for one row (all 32 lanes of the warp call it, `ok`
+// masks rows past the tile): v (and u, the up projection of GU) is the full
+// K reduction of sequence b.
+template <int B, int KIND>
+__device__ __forceinline__ void epi_final(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                          int s, int row, bool ok, int lane, const float (&v)[B],
+                                          const float (&u)[B]) {
+  float xn[B];
+  unsigned long long key[B];
+#pragma unroll
+  for (int b = 0; b < B; ++b) {
+    key[b] = 0ull;
+    xn[b] = 0.f;
+    if (!ok) continue;
+    // normed phases: the operand held x * gain, so the RMSNorm scale of
+    // sequence b multiplies the output column here
+    switch (KIND) {
+      case PH_QKV: p.qkv[b * p.qkv_rows + row] = v[b] * sm.inv[b]; break;
+      case PH_O:
+      case PH_DOWN: {
+        const float t = p.x[b * p.d + row] + v[b];
+        p.x[b * p.d + row] = t;
+        xn[b] = t;
+        break;
+      }
+      case PH_GU: {
+        const float g = v[b] * sm.inv[b], up = u[b] * sm.inv[b];
+        act_store1<B>(p.img_a, b, row, g / (1.0f + expf(-g)) * up);
+        if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_a, ph.R);
+        break;
+      }
+      case PH_LM: {
+        const float y = v[b] * sm.inv[b];
+        key[b] = argmax_key(y, (uint32_t)row);
+        if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = y;
+        break;
+      }
+      default: break;
+    }
+  }
+  if (KIND == PH_O || KIND == PH_DOWN) {
+    // the next normed phase's input: x * gain as an operand image, and the
+    // sums of squares of x over 8-row groups (fixed xor tree: independent of
+    // the grid); 8-row groups never straddle CTAs or row blocks
+    const uint16_t* gn =
+        (KIND == PH_O) ? p.w_layers + (uint64_t)ph.layer * p.layer_stride + p.off_gmlp
+        : (ph.layer + 1 < p.L) ? p.w_layers + (uint64_t)(ph.layer + 1) * p.layer_stride + p.off_gattn
+                               : p.g_final;
+    const float gr = ok ? bf16_bits_to_f32(gn[row]) : 0.f;
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      float t = xn[b] * xn[b];
+      t += __shfl_xor_sync(0xffffffffu, t, 1);
+      t += __shfl_xor_sync(0xffffffffu, t, 2);
+      t += __shfl_xor_sync(0xffffffffu, t, 4);
+      if (ok) {
+        if ((lane & 7) == 0) p.ssq[b * (p.d >> 3) + (row >> 3)] = t;
+        act_store1<B>(p.img_x, b, row, xn[b] * gr);
+        if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_x, ph.R);
+      }
+    }
+  }
+  if (KIND == PH_LM) {
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      unsigned long long kk = key[b];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long y = __shfl_xor_sync(0xffffffffu, kk, o);
+        kk = y > kk ? y : kk;
+      }
+      if (lane == 0 && kk) atomicMax(&sm.best[b], kk);
+    }
+  }
+}
+
+// partial of segment g, sequence b, at index idx (row, or 2 row + {0, 1} for GU)
+__device__ __forceinline__ float* kpart_at(const DecodeParams& p, const Phase& ph, int g, int b, int idx) {
+  const size_t rr = (size_t)ph.R * (ph.kind == PH_GU ? 2 : 1);
+  return p.kpart + ((size_t)g * p.B + b) * rr + idx;
+}
+
 template <int B, int KIND>
 __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm, const Phase& ph,
                                           int k, int s, int warp, int lane, uint32_t& tc,
@@ -480,9 +634,8 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
   constexpr int LO = decode_act_lo(B);
   constexpr bool gu = (KIND == PH_GU);
   const int q = warp & 3;
-  const bool first_seg = (ph.seg == 0), last_seg = (ph.seg == ph.nseg - 1);
   int r0, r1;
-  my_rows(ph.R, p.n_ctas, blockIdx.x, k, &r0, &r1);
+  piece_rows(ph, sm.span, p.n_ctas, blockIdx.x, k, &r0, &r1);
   for (int rt = r0; rt < r1; rt += kTileM) {
     const uint32_t slot = tc % kAccSlots, use = tc / kAccSlots;
     ++tc;
@@ -501,93 +654,144 @@ __device__ __forceinline__ void epi_phase(const DecodeParams& p, const Smem& sm,
     if (lane == 0) mbar_arrive(&sm.tempty[slot]);
     const int row = rt + 32 * q + lane;
     const bool ok = row < r1;
-    float v[B], u[B], xn[B];
+    float v[B], u[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
       v[b] = __uint_as_float(d0[b]) + __uint_as_float(d0[LO + b]);
       u[b] = gu ? __uint_as_float(d1[b]) + __uint_as_float(d1[LO + b]) : 0.f;
     }
-    unsigned long long key[B];
+    if (ph.nseg > 1) {   // (warp-uniform branches: the final epilogue uses shuffles)
+      if (ph.dist) {
+        // distributed: this piece's raw partial (summed by epi_finalize)
+        if (ok) {
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            if (gu) {
+              *reinterpret_cast<float2*>(kpart_at(p, ph, ph.seg, b, 2 * row)) = make_float2(v[b], u[b]);
+            } else {
+              *kpart_at(p, ph, ph.seg, b, row) = v[b];
+            }
+          }
+        }
+        continue;
+      }
+      // chained: the running sum ((p0 + p1) + ...) of this row's segments so
+      // far lives in slot 0 (written by this thread for the earlier segments)
+      if (ok) {
+        const int idx = gu ? 2 * row : row;
+#pragma unroll
+        for (int b = 0; b < B; ++b) {
+          float* acc = kpart_at(p, ph, 0, b, idx);
+          if (ph.seg > 0) {
+            v[b] += acc[0];
+            if (gu) u[b] += acc[1];
+          }
+          if (ph.seg < ph.nseg - 1) {
+            acc[0] = v[b];
+            if (gu) acc[1] = u[b];
+          }
+        }
+      }
+      if (ph.seg < ph.nseg - 1) continue;
+    }
+    epi_final<B, KIND>(p, sm, ph, s, row, ok, lane, v, u);
+  }
+}
+
+// Distributed multi-segment phases, the 4 epilogue warps after all of this
+// CTA's pieces: publish "my partials are stored" (a monotone per-CTA flag =
+// the phase's barrier target, release), then finish the row blocks this CTA
+// is assigned statically — block j goes to CTA floor(j C / nblk), so the
+// epilogue work is spread evenly — once the CTAs that computed the block's
+// pieces have published (acquire). A row's sum is ((p0 + p1) + p2) + ...,
+// the order of the chained mode, so the bits do not depend on the mode or on
+// which CTA computed a piece.
+__device__ __forceinline__ void st_release_u64(unsigned long long* a, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(a), "l"(v) : "memory");
+}
+
+// CTA owning group i of segment g (the c with T_c < end(g, i) <= T_{c+1},
+// T_c = floor(W c / C); see cta_span)
+__device__ __forceinline__ int group_owner(const Phase& ph, int C, int g, int i) {
+  const long long G8 = (ph.R + 7) >> 3;
+  const long long W = G8 * ph.KF;
+  const int wg = min(ph.w, ph.KF - g * ph.w);
+  const long long E = (long long)g * G8 * ph.w + (long long)(i + 1) * wg;
+  return (int)((E * C + W - 1) / W) - 1;
+}
+
+
+template <int B, int KIND>
+__device__ __forceinline__ void epi_finalize(const DecodeParams& p, const Smem& sm, const Phase& ph0,
+                                             int s, int warp, int lane, unsigned long long seq) {
+  constexpr bool gu = (KIND == PH_GU);
+  const int et = 32 * (warp & 3) + lane;
+  const int R = ph0.R, nseg = ph0.nseg, C = p.n_ctas, cta = blockIdx.x;
+  const int G8 = (R + 7) >> 3, nblk = (R + kFinRows - 1) / kFinRows;
+  named_bar_sync(2, 128);   // this CTA's partial stores are done (the release is cumulative)
+  if (et == 0) st_release_u64(p.pflag + cta, seq);
+  const int j0 = (int)(((long long)cta * nblk + C - 1) / C);
+  const int j1 = (int)(((long long)(cta + 1) * nblk + C - 1) / C);
+  for (int j = j0; j < j1; ++j) {
+    // thread g waits for the CTAs holding segment g's groups of block j
+    for (int g = et; g < nseg; g += 128) {
+      const int i0 = j * (kFinRows / 8), i1 = min(G8, (j + 1) * (kFinRows / 8)) - 1;
+      const int c0 = group_owner(ph0, C, g, i0), c1 = group_owner(ph0, C, g, i1);
+      for (int c = c0; c <= c1; ++c) {
+        if (c == cta) continue;
+        const uint64_t t0 = globaltimer();
+        while (ld_acquire_u64(p.pflag + c) < seq) {
+          if (ld_volatile_i32(p.err)) break;
+          if (globaltimer() - t0 > 4000000000ull) {
+            atomicExch(p.err, 1);
+            break;
+          }
+        }
+      }
+    }
+    named_bar_sync(2, 128);
+    const int row = j * kFinRows + et;   // warp q takes rows 32q.. of the block
+    const bool ok = row < R;
+    float v[B], u[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
-      key[b] = 0ull;
-      xn[b] = 0.f;
-      if (!ok) continue;
-      if (ph.nseg > 1) {
-        float* acc = p.kacc + (size_t)b * ph.R * (gu ? 2 : 1);
-        const int idx = gu ? 2 * row : row;
-        if (!first_seg) {
-          v[b] += acc[idx];
-          if (gu) u[b] += acc[idx + 1];
-        }
-        if (!last_seg) {
-          acc[idx] = v[b];
-          if (gu) acc[idx + 1] = u[b];
-          continue;
-        }
-      }
-      // normed phases: the operand held x * gain, so the RMSNorm scale of
-      // sequence b multiplies the output column here
-      switch (KIND) {
-        case PH_QKV: p.qkv[b * p.qkv_rows + row] = v[b] * sm.inv[b]; break;
-        case PH_O:
-        case PH_DOWN: {
-          const float t = p.x[b * p.d + row] + v[b];
-          p.x[b * p.d + row] = t;
-          xn[b] = t;
-          break;
-        }
-        case PH_GU: {
-          const float g = v[b] * sm.inv[b], up = u[b] * sm.inv[b];
-          act_store1<B>(p.img_a, b, row, g / (1.0f + expf(-g)) * up);
-          if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_a, ph.R);
-          break;
-        }
-        case PH_LM: {
-          const float y = v[b] * sm.inv[b];
-          key[b] = argmax_key(y, (uint32_t)row);
-          if (p.logits) p.logits[((size_t)(s - (p.P - 1)) * B + b) * p.V + row] = y;
-          break;
-        }
-        default: break;
-      }
+      v[b] = 0.f;
+      u[b] = 0.f;
     }
-    if ((KIND == PH_O || KIND == PH_DOWN) && last_seg) {
-      // the next normed phase's input: x * gain as an operand image, and the
-      // sums of squares of x over 8-row groups (fixed xor tree: independent of
-      // the grid); row groups never straddle CTAs (my_rows cuts at multiples of 8)
-      const uint16_t* gn =
-          (KIND == PH_O) ? p.w_layers + (uint64_t)ph.layer * p.layer_stride + p.off_gmlp
-          : (ph.layer + 1 < p.L) ? p.w_layers + (uint64_t)(ph.layer + 1) * p.layer_stride + p.off_gattn
-                                 : p.g_final;
-      const float gr = ok ? bf16_bits_to_f32(gn[row]) : 0.f;
+    if (ok) {
+      // partials in segment order, two segments' loads in flight at a time
+      for (int g0 = 0; g0 < nseg; g0 += 2) {
+        float tv[2][B], tu[2][B];
 #pragma unroll
-      for (int b = 0; b < B; ++b) {
-        float t = xn[b] * xn[b];
-        t += __shfl_xor_sync(0xffffffffu, t, 1);
-        t += __shfl_xor_sync(0xffffffffu, t, 2);
-        t += __shfl_xor_sync(0xffffffffu, t, 4);
-        if (ok) {
-          if ((lane & 7) == 0) p.ssq[b * (p.d >> 3) + (row >> 3)] = t;
-          act_store1<B>(p.img_x, b, row, xn[b] * gr);
-          if (b == 0 && row == ph.R - 1) img_zero_tail<B>(p.img_x, ph.R);
+        for (int t = 0; t < 2; ++t) {
+#pragma unroll
+          for (int b = 0; b < B; ++b) {
+            tv[t][b] = tu[t][b] = 0.f;
+            if (g0 + t < nseg) {
+              if (gu) {
+                const float2 x2 = __ldcg(reinterpret_cast<const float2*>(kpart_at(p, ph0, g0 + t, b, 2 * row)));
+                tv[t][b] = x2.x;
+                tu[t][b] = x2.y;
+              } else {
+                tv[t][b] = __ldcg(kpart_at(p, ph0, g0 + t, b, row));
+              }
+            }
+          }
+        }
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+          if (g0 + t < nseg) {
+#pragma unroll
+            for (int b = 0; b < B; ++b) {
+              v[b] = (g0 + t == 0) ? tv[t][b] : tv[t][b] + v[b];
+              u[b] = (g0 + t == 0) ? tu[t][b] : tu[t][b] + u[b];
+            }
+          }
         }
       }
     }
-    if (KIND == PH_LM && last_seg) {
-#pragma unroll
-      for (int b = 0; b < B; ++b) {
-        unsigned long long kk = key[b];
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          const unsigned long long y = __shfl_xor_sync(0xffffffffu, kk, o);
-          kk = y > kk ? y : kk;
-        }
-        if (lane == 0 && kk) atomicMax(&sm.best[b], kk);
-      }
-    }
+    epi_final<B, KIND>(p, sm, ph0, s, row, ok, lane, v, u);
   }
-  if (KIND == PH_O || KIND == PH_DOWN || KIND == PH_GU) fence_proxy_async_global();
 }
 
 template <int B>
@@ -601,6 +805,20 @@ __device__ __forceinline__ void epi_dispatch(const DecodeParams& p, const Smem& 
     case PH_DOWN: epi_phase<B, PH_DOWN>(p, sm, ph, k, s, warp, lane, tc, tmem_base, w_tf); break;
     default: epi_phase<B, PH_LM>(p, sm, ph, k, s, warp, lane, tc, tmem_base, w_tf); break;
   }
+}
+
+// All segments of a phase done: finish multi-segment rows, then make the
+// operand images written here visible to the next phase's bulk copies.
+template <int B>
+__device__ __forceinline__ void epi_close(const DecodeParams& p, const Smem& sm, const Phase& ph0,
+                                          int s, int warp, int lane, unsigned long long seq) {
+  if (ph0.dist) {   // only O and DOWN phases are distributed (make_phase)
+    if (ph0.kind == PH_O)
+      epi_finalize<B, PH_O>(p, sm, ph0, s, warp, lane, seq);
+    else
+      epi_finalize<B, PH_DOWN>(p, sm, ph0, s, warp, lane, seq);
+  }
+  if (ph0.kind == PH_O || ph0.kind == PH_DOWN || ph0.kind == PH_GU) fence_proxy_async_global();
 }
 
 // ---------------------------------------------------------------------------
@@ -811,6 +1029,7 @@ __device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer
 // item by item) and the fused-attention O input (computed into the operand).
 // ---------------------------------------------------------------------------
 constexpr int kCache = 2;
+constexpr int kDecodeTl = 2560;   // timeline words in the profile buffer (after [n_ctas][16])
 
 // Fixed-order RMSNorm reduction of the per-thread partials acc[b]: warp
 // shuffle trees, then warps in order; sm.inv[b] = 1 / sqrt(mean + eps).
@@ -879,15 +1098,15 @@ __device__ __forceinline__ void issue_img_copy(const DecodeParams& p, const Smem
 
 template <int B>
 __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm, const Phase& ph,
-                                          int s, int tid_c) {
+                                          int s, int tid_c, bool prologue, bool fill) {
   const int kind = ph.kind, layer = ph.layer;
   const int cta = blockIdx.x, C = p.n_ctas;
   const int warp = tid_c >> 5, lane = tid_c & 31;
   constexpr int LO = decode_act_lo(B);
   const int K = ph.K, k0 = ph.k0, KF = ph.KF;
   const int nq = ph.nkb * 8;            // 16-byte chunks per operand row
-  if (ph.seg > 0) named_bar_sync(1, kNCT);   // the previous segment's MMAs have completed
-  if (kind == PH_LM && ph.seg == 0 && tid_c < B) sm.best[tid_c] = 0ull;
+  if (!prologue) named_bar_sync(1, kNCT);   // the previous segment's MMAs have completed
+  if (kind == PH_LM && prologue && tid_c < B) sm.best[tid_c] = 0ull;
   if (kind == PH_O && p.fuse_att) {
     // every CTA computes all heads (small attention): o lands in the operand
     for (int i = tid_c; i < B * nq; i += kNCT) {
@@ -907,7 +1126,7 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
     return;
   }
   // --- layer-0 QKV: embedding rows of the step's tokens ---------------------
-  if (ph.seg == 0) {
+  if (prologue) {
     // input token: prompt for s < P, else the argmax of step s-1 (reduced from
     // the per-CTA candidates, identically in every CTA).
     if (tid_c < B) {
@@ -938,7 +1157,7 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
   };
   const int n_items = B * nq;
   // single pass: the whole input is this segment and fits the register cache
-  const bool cached = (ph.nseg == 1) && (n_items <= kCache * kNCT);
+  const bool cached = fill && (ph.nseg == 1) && (n_items <= kCache * kNCT);
   float cv[kCache][8];
   if (cached) {
 #pragma unroll
@@ -953,7 +1172,7 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
       }
     }
   }
-  if (ph.seg == 0) {
+  if (prologue) {
     // RMSNorm over the FULL input (normalise, then scale; eps inside the sqrt)
     float acc[B];
 #pragma unroll
@@ -994,13 +1213,28 @@ __device__ __forceinline__ void stage_act(const DecodeParams& p, const Smem& sm,
       }
     }
     norm_finish<B>(p, sm, acc, KF, tid_c);
+    // the residual stream x = the embedding rows (CTA 0, every column; a
+    // single-segment phase writes it while staging)
+    if (cta == 0 && ph.nseg > 1) {
+      for (int i = tid_c; i < B * (KF / 8); i += kNCT) {
+        const int b = i / (KF / 8), col = (i % (KF / 8)) * 8;
+        float f[8];
+        load8(b, col, f);
+        *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col) = make_float4(f[0], f[1], f[2], f[3]);
+        *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col + 4) = make_float4(f[4], f[5], f[6], f[7]);
+      }
+    }
+    if (!fill) {
+      named_bar_sync(1, kNCT);
+      return;
+    }
   }
-  // x (CTA 0), gain-scaled operand split hi/lo; columns >= K are zero
+  // gain-scaled operand split hi/lo; columns >= K are zero
   auto put = [&](int i, float (&f)[8]) {
     const int b = i / nq, q = i - b * nq;
     const int col = k0 + q * 8;
     if (q * 8 < K) {
-      if (cta == 0) {
+      if (cta == 0 && ph.nseg == 1) {
         *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col) = make_float4(f[0], f[1], f[2], f[3]);
         *reinterpret_cast<float4*>(p.x + (size_t)b * p.d + col + 4) = make_float4(f[4], f[5], f[6], f[7]);
       }
@@ -1067,6 +1301,10 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     fence_mbar_init();
     if (blockIdx.x == 0) p.stamps[0] = globaltimer();
   }
+  if (threadIdx.x >= 32 && threadIdx.x < 32 + 6 && threadIdx.x - 32 != PH_ATT) {
+    const Phase ph = make_phase<B>(p, (int)threadIdx.x - 32, 0, 0);
+    if (ph.dist) cta_span(ph, p.n_ctas, blockIdx.x, sm.span + 4 * ph.kind);
+  }
   // operand rows of absent sequences stay zero for the whole launch
   const int act_chunks = decode_act_bytes(B, kmax) / 16;
   for (int i = threadIdx.x; i < act_chunks; i += blockDim.x)
@@ -1095,35 +1333,55 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
     for (int k = 0; k < nph; ++k) {
       const int kind = phase_kind(k, L, p.fuse_att);
       const int layer = k / pl;
+#ifdef MX_PROF_BUCKETS
+      // timeline (globaltimer) of the phases of layer L/2 at step S/2, per CTA:
+      // [0] start [1] operand ready [2] last MMA issued / attention done
+      // [3] epilogue done (warp 2) [4] barrier arrive [5] barrier exit
+      unsigned long long* tl =
+          (p.prof && s == S / 2 && layer == L / 2 && kind != PH_LM)
+              ? p.prof + kDecodeTl + ((size_t)blockIdx.x * 5 + (k % pl)) * 6 : nullptr;
+#else
+      unsigned long long* tl = nullptr;
+#endif
+      if (tl && tid_c == 0) tl[0] = globaltimer();
       long long t0 = MX_CLK();
       if (kind == PH_ATT) {
         attention_phase<B>(p, sm, layer, s, tid_c);
+        if (tl && tid_c == 0) tl[1] = tl[2] = globaltimer();
         const long long t1 = MX_CLK();
         c_att += t1 - t0;
         t0 = t1;
       } else {
         const int nseg = phase_segments<B>(p, kind);
+        const Phase ph0 = make_phase<B>(p, kind, layer, 0);
+        // this CTA's segments [ga, gb] (contiguous; empty when ga > gb); a
+        // single-segment phase is staged even by a CTA without rows
+        const int ga = ph0.dist ? sm.span[4 * kind] : 0;
+        const int gb = ph0.dist ? sm.span[4 * kind + 2] : nseg - 1;
+        const int n_act = gb - ga + 1 > 0 ? gb - ga + 1 : 0;
         if (img_phase(p, kind, layer)) {
-          // segment s + 1's operand is copied into one half while the MMAs of
-          // segment s read the other (kStageWarp lane 0 runs the copies)
+          // the operand of this CTA's next segment is copied into one half while
+          // the MMAs of its current segment read the other (kStageWarp lane 0
+          // runs the copies)
           const uint32_t img0 = img_seq;
-          img_seq += (uint32_t)nseg;
+          img_seq += (uint32_t)n_act;
           const bool stager = (warp_id == kStageWarp);   // lane 0 issues, the warp stays converged
-          auto half = [&](int seg) { return nseg == 1 ? 0u : (img0 + (uint32_t)seg) & 1u; };
+          auto half = [&](int seg) { return nseg == 1 ? 0u : (img0 + (uint32_t)(seg - ga)) & 1u; };
           auto copy_seg = [&](int seg) {
             const uint32_t hb = half(seg);
             if (lane == 0) issue_img_copy<B>(p, sm, make_phase<B>(p, kind, layer, seg), hb, act_use[hb]);
             ++act_use[hb];
             __syncwarp();
           };
-          if (stager) copy_seg(0);
-          prep_img<B>(p, sm, make_phase<B>(p, kind, layer, 0), tid_c);
+          if (stager && n_act > 0) copy_seg(ga);
+          prep_img<B>(p, sm, ph0, tid_c);
+          if (tl && tid_c == 0) tl[1] = globaltimer();
           const long long t1 = MX_CLK();
           c_stage += t1 - t0;
           if (stager) {
-            for (int seg = 1; seg < nseg; ++seg) copy_seg(seg);
+            for (int seg = ga + 1; seg <= gb; ++seg) copy_seg(seg);
           } else if (warp_id == kMmaWarp) {
-            for (int seg = 0; seg < nseg; ++seg) {
+            for (int seg = ga; seg <= gb; ++seg) {
               const Phase ph = make_phase<B>(p, kind, layer, seg);
               const uint32_t hb = half(seg);
               const long long tw = MX_CLK();
@@ -1136,18 +1394,25 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
                            hb * (uint32_t)(decode_act_bytes(B, decode_seg_cols(B)) / 2));
               umma_commit_warp(smem_u32(&sm.actfree[hb]));   // half free once these MMAs completed
             }
+            if (tl && lane == 0) tl[2] = globaltimer();
           } else if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
-            for (int seg = 0; seg < nseg; ++seg)
+            for (int seg = ga; seg <= gb; ++seg)
               epi_dispatch<B>(p, sm, make_phase<B>(p, kind, layer, seg), k, s, warp_id, lane, tc,
                               tmem_base, w_tf);
+            epi_close<B>(p, sm, ph0, s, warp_id, lane, target + (unsigned long long)p.n_ctas);
+            if (tl && tid_c == 32) tl[3] = globaltimer();
           }
           const long long t2 = MX_CLK();
           c_gemv += t2 - t1;
           t0 = t2;
         } else {
-          for (int seg = 0; seg < nseg; ++seg) {
+          // layer-0 QKV (embedding rows) or the fused-attention O phase (never
+          // distributed: every CTA runs all segments, so the prologue — input
+          // tokens, RMSNorm / attention — runs everywhere)
+          for (int seg = ga; seg <= gb; ++seg) {
             const Phase ph = make_phase<B>(p, kind, layer, seg);
-            stage_act<B>(p, sm, ph, s, tid_c);
+            stage_act<B>(p, sm, ph, s, tid_c, seg == ga, true);
+            if (tl && tid_c == 0 && seg == ga) tl[1] = globaltimer();
             const long long t1 = MX_CLK();
             if (kind == PH_O && p.fuse_att)
               c_att += t1 - t0;
@@ -1155,12 +1420,17 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
               c_stage += t1 - t0;
             if (warp_id == kMmaWarp) {
               mma_phase<B>(p, sm, ph, k, stage, phase_bit, n_stages, tc, tmem_base, w_full, w_acc);
+              if (tl && lane == 0) tl[2] = globaltimer();
             } else if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
               epi_dispatch<B>(p, sm, ph, k, s, warp_id, lane, tc, tmem_base, w_tf);
             }
             const long long t2 = MX_CLK();
             c_gemv += t2 - t1;
             t0 = t2;
+          }
+          if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
+            epi_close<B>(p, sm, ph0, s, warp_id, lane, target + (unsigned long long)p.n_ctas);
+            if (tl && tid_c == 32) tl[3] = globaltimer();
           }
         }
         if (kind == PH_LM) {
@@ -1169,7 +1439,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
         }
       }
       target += (unsigned long long)p.n_ctas;
-      grid_barrier(p, target, tid_c);
+      grid_barrier(p, target, tid_c, tl);
       c_bar += MX_CLK() - t0;
     }
   }

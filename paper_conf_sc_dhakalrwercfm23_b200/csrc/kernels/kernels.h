@@ -61,6 +61,26 @@ MX_HD constexpr int decode_act_bytes(int B, int kmax) {
           kBlkK) *
          decode_act_blk_bytes(B);
 }
+// K segments of one GEMV phase (R output rows, KF input columns), a function
+// of the shape only, so results stay bit-identical for any partition size:
+// one segment when the input fits the operand region, else segments of at
+// most half of it (the operand of segment s + 1 is copied into one half while
+// the MMAs of segment s read the other). Large matrices (R x KF >= 2^24, e.g.
+// every 7B phase) are split into half-region segments even when the input
+// fits: their (segment, row-group) pieces are spread over the CTAs, so a CTA
+// issues each M = 128 MMA on ~2x more of its own rows than a pure row split
+// would give it (a skinny MMA costs the same issue time for 8 or 128 rows).
+MX_HD constexpr int decode_nseg(int B, long long R, int KF, int splittable) {
+  return KF > decode_seg_cols(B)
+             ? (KF + decode_seg_cols(B) / 2 - 1) / (decode_seg_cols(B) / 2)
+         : (splittable && R * KF >= (1ll << 24) && KF > decode_seg_cols(B) / 2)
+             ? (KF + decode_seg_cols(B) / 2 - 1) / (decode_seg_cols(B) / 2)
+             : 1;
+}
+// Rows per finalisation block of a distributed multi-segment phase: one CTA
+// (assigned statically) sums the block's segment partials in segment order
+// and applies the phase's epilogue.
+constexpr int kFinRows = 128;
 // Bytes of a global image of the activation operand over `cols` input columns
 // (the shared-memory layout above, every 64-column block): the phase that
 // produces an input writes it in this form, the consuming phase copies each
@@ -98,7 +118,8 @@ struct DecodeParams {
   uint8_t* img_a;
   float* ssq;                // [B][d / 8] sums of squares of x over 8-row groups
   unsigned long long* cand;  // [kMaxCtas][B] per-CTA argmax keys
-  float* kacc;               // split-K partial sums [B][2 * max(qkv_rows, ff, d, V)]
+  float* kpart;              // segment partial sums [nseg][B][R (x2 for gate/up)] (decode_kpart_floats)
+  unsigned long long* pflag; // [kMaxCtas] per-CTA "partials stored" flags (monotone: barrier targets)
   uint16_t* kc;              // [L][B][Hkv][max_seq][hd] bf16
   uint16_t* vc;
   const int* prompt;         // [B][P] (host-mapped)
@@ -117,6 +138,8 @@ struct DecodeParams {
   int inject_err;            // test hook (mx_debug_inject_error): reported as the task's device error
 };
 
+// Floats of the segment-partial buffer for a shape (max over the phases).
+uint64_t decode_kpart_floats(int B, int d, int q_dim, int qkv_rows, int ff, int V, int fuse_att);
 // 1 if every CTA computes the whole attention itself (B*H*hd <= 1024, grid small enough).
 int decode_fuse_attention(int B, int H, int hd, int n_ctas);
 // 1 if this build records the per-CTA cycle buckets (-DMX_PROF_BUCKETS).

@@ -163,8 +163,8 @@ static int validate_fn(const mx_fn_desc& d) {
       set_error("decode cfg: max_seq <= %d and 1 <= max_batch <= 8", mxk::kMaxSeqCap);
       return MX_EINVAL;
     }
-    if (c.d_model > 8192 || c.d_ff > 16384 || q > 16384) {
-      set_error("decode cfg: d_model <= 8192, q_dim and d_ff <= 16384");
+    if (c.d_model > 8192 || c.d_ff > 16384 || q > 16384 || c.vocab > (1 << 20)) {
+      set_error("decode cfg: d_model <= 8192, q_dim and d_ff <= 16384, vocab <= 2^20");
       return MX_EINVAL;
     }
     const int kmax = std::max(std::max(c.d_model, q), c.d_ff);
@@ -498,8 +498,14 @@ static int alloc_decode_slot(Partition& p, FnInst& fi, Slot& s) {
   if ((rc = alloc_ptr(p, mxk::decode_img_bytes(8, (int)ff), &s.img_a))) return rc;
   if ((rc = alloc_ptr(p, B * (d / 8) * 4, &s.ssq))) return rc;
   if ((rc = alloc_ptr(p, (uint64_t)mxk::kMaxCtas * B * 8, &s.cand))) return rc;
-  const uint64_t kacc_rows = std::max(std::max(q + 2 * kv, 2 * ff), std::max(d, V));
-  if ((rc = alloc_ptr(p, B * kacc_rows * 4, &s.kacc))) return rc;
+  // segment partials of multi-segment phases (any batch up to max_batch) and
+  // the row-block arrival counters that finish them
+  uint64_t kpart = 0;
+  for (uint64_t b = 1; b <= B; ++b)
+    kpart = std::max(kpart, mxk::decode_kpart_floats((int)b, (int)d, (int)q, (int)(q + 2 * kv),
+                                                     (int)ff, (int)V, 0));
+  if ((rc = alloc_ptr(p, std::max<uint64_t>(kpart, 64) * 4, &s.kpart))) return rc;
+  if ((rc = alloc_ptr(p, (uint64_t)mxk::kMaxCtas * 8, &s.pflag))) return rc;
   if ((rc = alloc_ptr(p, L * B * kv * T * 2, &s.kc))) return rc;
   if ((rc = alloc_ptr(p, L * B * kv * T * 2, &s.vc))) return rc;
   if ((rc = alloc_ptr(p, B * T * 4, &s.prompt))) return rc;
@@ -776,7 +782,8 @@ static int load_instance(Gpu& gpu, Partition& p, Fn& fn, FnInst** out) {
       // sequences are never written by the kernel and must read as zero
       const mx_decode_cfg& c = d.dec;
       const int q = c.n_heads * c.head_dim;
-      if (drv().cuMemsetD8Async(s.img_x, 0, mxk::decode_img_bytes(8, c.d_model), st) != CUDA_SUCCESS ||
+      if (drv().cuMemsetD8Async(s.pflag, 0, (size_t)mxk::kMaxCtas * 8, st) != CUDA_SUCCESS ||
+          drv().cuMemsetD8Async(s.img_x, 0, mxk::decode_img_bytes(8, c.d_model), st) != CUDA_SUCCESS ||
           drv().cuMemsetD8Async(s.img_o, 0, mxk::decode_img_bytes(8, q), st) != CUDA_SUCCESS ||
           drv().cuMemsetD8Async(s.img_a, 0, mxk::decode_img_bytes(8, c.d_ff), st) != CUDA_SUCCESS) {
         set_error("slot reset failed");
@@ -839,6 +846,7 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
   CUevent* ev = e->ev[t->lane];
   if (s.need_reset) {
     if (s.bar) CU_TRY(drv().cuMemsetD8Async(s.bar, 0, 8, st));
+    if (s.pflag) CU_TRY(drv().cuMemsetD8Async(s.pflag, 0, (size_t)mxk::kMaxCtas * 8, st));
     CU_TRY(drv().cuMemsetD8Async(s.stamps, 0, 64, st));
     s.bar_count = 0;
     s.need_reset = false;
@@ -899,7 +907,8 @@ static int launch_task(Gpu& gpu, Partition& p, Task* t) {
     k.img_a = reinterpret_cast<uint8_t*>(s.img_a);
     k.ssq = reinterpret_cast<float*>(s.ssq);
     k.cand = reinterpret_cast<unsigned long long*>(s.cand);
-    k.kacc = reinterpret_cast<float*>(s.kacc);
+    k.kpart = reinterpret_cast<float*>(s.kpart);
+    k.pflag = reinterpret_cast<unsigned long long*>(s.pflag);
     k.kc = reinterpret_cast<uint16_t*>(s.kc);
     k.vc = reinterpret_cast<uint16_t*>(s.vc);
     k.prompt = reinterpret_cast<const int*>(s.d_in);

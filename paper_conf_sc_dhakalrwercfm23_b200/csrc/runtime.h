@@ -87,7 +87,7 @@ struct Task {
 struct Slot {
   bool busy = false;
   // decode
-  CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kacc = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
+  CUdeviceptr x = 0, qkv = 0, o = 0, a = 0, cand = 0, kpart = 0, pflag = 0, kc = 0, vc = 0, prompt = 0, tokens = 0,
               logits = 0, img_x = 0, img_o = 0, img_a = 0, ssq = 0;
   // mpnn: device image of a task's packed inputs (Task::blob)
   CUdeviceptr in_blob = 0;

@@ -57,5 +57,24 @@ if os.environ.get("MX_DECODE_PROF") == "1":
     for i, nm in names.items():
         print(f"  {nm:16s} mean {pr[:, i].mean() / 1e6:9.2f} Mcyc  ({pr[:, i].mean() / tot * 100:5.1f}%)"
               f"  min {pr[:, i].min() / 1e6:8.2f} max {pr[:, i].max() / 1e6:8.2f}")
+    # timeline of layer L/2 at step S/2 (globaltimer ns, words 2560.. of the buffer)
+    import numpy as np
+    full = mx.decode_profile(p, 1024).reshape(-1).astype(np.int64)
+    tl = full[2560:2560 + n * 5 * 6].reshape(n, 5, 6)
+    base = tl[:, 0, 0][tl[:, 0, 0] > 0].min() if (tl[:, 0, 0] > 0).any() else 0
+    print("timeline (us from the first phase start; median/max over CTAs)")
+    print("  ph  start(min..max)   ready-start  mma_end(med/max)  epi_end(med/max)  arrive(min..max)"
+          "  exit(min..max)  exit-lastarrive")
+    for ph in range(5):
+        t = tl[:, ph, :].astype(float)
+        if not (t[:, 0] > 0).any():
+            continue
+        r = (t - base) / 1e3
+        arr, ex = r[:, 4], r[:, 5]
+        print(f"  {ph}  {r[:, 0].min():7.2f}..{r[:, 0].max():7.2f}  {np.median(r[:, 1] - r[:, 0]):6.2f}"
+              f"  {np.median(r[:, 2]):7.2f}/{r[:, 2].max():7.2f}  {np.median(r[:, 3]):7.2f}/{r[:, 3].max():7.2f}"
+              f"  {arr.min():7.2f}..{arr.max():7.2f}  {ex.min():7.2f}..{ex.max():7.2f}  {ex.min() - arr.max():6.2f}")
+    os.makedirs("gpurun_out", exist_ok=True)
+    np.save(os.environ.get("MX_TL_OUT", f"gpurun_out/tl_{a.cfg}_{a.sms}sm_b{a.batch}.npy"), tl)
 mx.part_destroy(p)
 mx.mx_shutdown()
