@@ -1000,17 +1000,246 @@ __device__ __forceinline__ void attend(const DecodeParams& p, const Smem& sm, in
   }
 }
 
-// Separate attention phase (large attention): items spread over all warps of all CTAs.
+// ---------------------------------------------------------------------------
+// Separate attention phase, key-block split (flash-decoding inside a CTA):
+// item (b, h) goes to CTA (b H + h) mod C; its keys are cut into blocks of KB
+// positions, one warp computes one block's softmax partial (block max m_i,
+// sum l_i of exp(s - m_i), exp-weighted values a_i) into shared memory, and
+// one warp folds the partials in block order (M' = max(M, m_i), rescale by
+// exp(M - M') / exp(m_i - M')). The blocks and the fold order depend only on
+// t and the shape, so the result does not depend on the partition size.
+// ---------------------------------------------------------------------------
+template <int B, int HD>
+__device__ __forceinline__ void att_block(const DecodeParams& p, const Smem& sm, int layer, int t,
+                                          int b, int h, int m, bool writer, int warp, int lane,
+                                          float* part) {
+  constexpr int HALF = HD / 2;
+  constexpr int PPL = (HALF + 31) / 32;       // rope pairs per lane
+  constexpr int KB = (HD <= 64) ? 32 : 16;    // keys per block
+  constexpr int LPK = 32 / KB;                // lanes per key
+  constexpr int KSEG = HD / LPK;              // key elements per lane
+  constexpr int KV4 = KSEG / 8;               // 16-byte loads per lane per key
+  constexpr int DPL = HD / 32;                // output dims per lane
+  const int Hkv = p.Hkv;
+  const int kvh = h / (p.H / Hkv);
+  float* qs = sm.att + warp * 3 * kAttHd;
+  float* ks = qs + kAttHd;
+  float* vs = ks + kAttHd;
+  const float* base = p.qkv + (size_t)b * p.qkv_rows;
+  const size_t cache_row0 = ((((size_t)layer * B + b) * Hkv + kvh) * p.max_seq) * HD;
+  uint16_t* kcache = p.kc + cache_row0;
+  uint16_t* vcache = p.vc + cache_row0;
+  const int kslot = lane / LPK, kseg = (lane % LPK) * KSEG;
+  const int j = m * KB + kslot;
+  const bool cur = (t / KB == m);   // this block holds the current token
+  // the block's cached keys / values (independent of the current token)
+  uint4 kr[KV4];
+#pragma unroll
+  for (int i = 0; i < KV4; ++i)
+    kr[i] = (j < t) ? *reinterpret_cast<const uint4*>(kcache + (size_t)j * HD + kseg + 8 * i)
+                    : make_uint4(0, 0, 0, 0);
+  uint32_t vv[KB][(DPL + 1) / 2];
+#pragma unroll
+  for (int jj = 0; jj < KB; ++jj) {
+    const int jk = m * KB + jj;
+    const uint16_t* src = vcache + (size_t)jk * HD + lane * DPL;
+    if (DPL == 4) {
+      uint2 v2 = make_uint2(0u, 0u);
+      if (jk < t) v2 = *reinterpret_cast<const uint2*>(src);
+      vv[jj][0] = v2.x;
+      vv[jj][(DPL + 1) / 2 - 1] = v2.y;
+    } else if (DPL == 2) {
+      vv[jj][0] = (jk < t) ? *reinterpret_cast<const uint32_t*>(src) : 0u;
+    } else {
+      vv[jj][0] = (jk < t) ? (uint32_t)*src : 0u;
+    }
+  }
+  // RoPE(q) at position t (every block), RoPE(k) / v of the current token
+  // (its block only; the cache row is written once per kv head)
+#pragma unroll
+  for (int pi = 0; pi < PPL; ++pi) {
+    const int i = lane + 32 * pi;
+    if (i < HALF) {
+      const float c = p.rope_cs[((size_t)t * HALF + i) * 2 + 0];
+      const float sn = p.rope_cs[((size_t)t * HALF + i) * 2 + 1];
+      const float q1 = base[h * HD + i], q2 = base[h * HD + i + HALF];
+      qs[i] = q1 * c - q2 * sn;
+      qs[i + HALF] = q2 * c + q1 * sn;
+      if (cur) {
+        const float* kb = base + p.q_dim + kvh * HD;
+        const float k1 = kb[i], k2 = kb[i + HALF];
+        const float* vb = base + p.q_dim + p.kv_dim + kvh * HD;
+        const uint16_t kb1 = f32_to_bf16_rne(k1 * c - k2 * sn);
+        const uint16_t kb2 = f32_to_bf16_rne(k2 * c + k1 * sn);
+        const uint16_t vb1 = f32_to_bf16_rne(vb[i]);
+        const uint16_t vb2 = f32_to_bf16_rne(vb[i + HALF]);
+        ks[i] = bf16_bits_to_f32(kb1);
+        ks[i + HALF] = bf16_bits_to_f32(kb2);
+        vs[i] = bf16_bits_to_f32(vb1);
+        vs[i + HALF] = bf16_bits_to_f32(vb2);
+        if (writer) {
+          kcache[(size_t)t * HD + i] = kb1;
+          kcache[(size_t)t * HD + i + HALF] = kb2;
+          vcache[(size_t)t * HD + i] = vb1;
+          vcache[(size_t)t * HD + i + HALF] = vb2;
+        }
+      }
+    }
+  }
+  __syncwarp();
+  float dot = 0.f;
+  if (j < t) {
+#pragma unroll
+    for (int i = 0; i < KV4; ++i) {
+      float kf[8];
+      unpack8(kr[i], kf);
+      const float4 qa = *reinterpret_cast<const float4*>(qs + kseg + 8 * i);
+      const float4 qb = *reinterpret_cast<const float4*>(qs + kseg + 8 * i + 4);
+      dot = fmaf(qa.x, kf[0], dot);
+      dot = fmaf(qa.y, kf[1], dot);
+      dot = fmaf(qa.z, kf[2], dot);
+      dot = fmaf(qa.w, kf[3], dot);
+      dot = fmaf(qb.x, kf[4], dot);
+      dot = fmaf(qb.y, kf[5], dot);
+      dot = fmaf(qb.z, kf[6], dot);
+      dot = fmaf(qb.w, kf[7], dot);
+    }
+  } else if (j == t) {
+#pragma unroll 4
+    for (int e = 0; e < KSEG; e += 4) {
+      const float4 qa = *reinterpret_cast<const float4*>(qs + kseg + e);
+      const float4 ka = *reinterpret_cast<const float4*>(ks + kseg + e);
+      dot = fmaf(qa.x, ka.x, dot);
+      dot = fmaf(qa.y, ka.y, dot);
+      dot = fmaf(qa.z, ka.z, dot);
+      dot = fmaf(qa.w, ka.w, dot);
+    }
+  }
+  if (LPK == 2) dot += __shfl_xor_sync(0xffffffffu, dot, 1);
+  const float sc = (j <= t) ? dot / sqrtf((float)HD) : -FLT_MAX;
+  const float bm = warp_max(sc);
+  const float ej = (j <= t) ? expf(sc - bm) : 0.f;
+  const float l = warp_sum((lane % LPK) == 0 ? ej : 0.f);
+  float acc[DPL];
+#pragma unroll
+  for (int d = 0; d < DPL; ++d) acc[d] = 0.f;
+#pragma unroll
+  for (int jj = 0; jj < KB; ++jj) {
+    const int jk = m * KB + jj;
+    const float e = __shfl_sync(0xffffffffu, ej, jj * LPK);
+    float v[4];
+    if (jk == t) {
+#pragma unroll
+      for (int d = 0; d < 4; ++d) v[d] = (d < DPL) ? vs[lane * DPL + d] : 0.f;
+    } else {
+      v[0] = __uint_as_float(vv[jj][0] << 16);
+      v[1] = __uint_as_float(vv[jj][0] & 0xffff0000u);
+      v[2] = __uint_as_float(vv[jj][(DPL + 1) / 2 - 1] << 16);
+      v[3] = __uint_as_float(vv[jj][(DPL + 1) / 2 - 1] & 0xffff0000u);
+    }
+#pragma unroll
+    for (int d = 0; d < DPL; ++d) acc[d] = fmaf(e, v[d], acc[d]);
+  }
+#pragma unroll
+  for (int d = 0; d < DPL; ++d) part[lane * DPL + d] = acc[d];
+  if (lane == 0) {
+    part[HD] = bm;
+    part[HD + 1] = l;
+  }
+  __syncwarp();
+}
+
+// Fold of one item's block partials (block order) -> o_h in the O phase's image.
+template <int B, int HD>
+__device__ __forceinline__ void att_fold(const DecodeParams& p, int b, int h, int nb,
+                                         const float* part, int lane) {
+  constexpr int DPL = HD / 32;
+  float M = -FLT_MAX, L = 0.f, acc[DPL];
+#pragma unroll
+  for (int d = 0; d < DPL; ++d) acc[d] = 0.f;
+  for (int m = 0; m < nb; ++m) {
+    const float* pm = part + m * (HD + 2);
+    const float mi = pm[HD], li = pm[HD + 1];
+    const float Mn = fmaxf(M, mi);
+    const float sa = expf(M - Mn), sb = expf(mi - Mn);
+    L = L * sa + li * sb;
+#pragma unroll
+    for (int d = 0; d < DPL; ++d) acc[d] = acc[d] * sa + pm[lane * DPL + d] * sb;
+    M = Mn;
+  }
+#pragma unroll
+  for (int d = 0; d < DPL; ++d) {
+    const int dd = lane * DPL + d;
+    act_store1<B>(p.img_o, b, h * HD + dd, acc[d] / L);
+    if (b == 0 && h * HD + dd == p.q_dim - 1) img_zero_tail<B>(p.img_o, p.q_dim);
+  }
+}
+
+template <int B, int HD>
+__device__ __forceinline__ void attention_split(const DecodeParams& p, const Smem& sm, int layer,
+                                                int t, int tid_c, float* part_base, int avail) {
+  constexpr int KB = (HD <= 64) ? 32 : 16;
+  constexpr int PW = HD + 2;
+  const int warp = tid_c >> 5, lane = tid_c & 31;
+  const int C = p.n_ctas, cta = blockIdx.x, items = B * p.H, group = p.H / p.Hkv;
+  const int nb = t / KB + 1;
+  const int slots = avail / (nb * PW);
+  const int n_my = (cta < items) ? (items - cta + C - 1) / C : 0;
+  for (int i0 = 0; i0 < n_my; i0 += slots) {
+    const int ni = min(slots, n_my - i0);
+    for (int task = warp; task < ni * nb; task += kConsumerWarps) {
+      const int sl = task / nb, m = task - sl * nb;
+      const int it = cta + (i0 + sl) * C;
+      const int b = it / p.H, h = it - b * p.H;
+      att_block<B, HD>(p, sm, layer, t, b, h, m, (h % group) == 0, warp, lane,
+                       part_base + (size_t)(sl * nb + m) * PW);
+    }
+    named_bar_sync(1, kNCT);
+    for (int sl = warp; sl < ni; sl += kConsumerWarps) {
+      const int it = cta + (i0 + sl) * C;
+      const int b = it / p.H, h = it - b * p.H;
+      att_fold<B, HD>(p, b, h, nb, part_base + (size_t)sl * nb * PW, lane);
+    }
+    named_bar_sync(1, kNCT);   // the partial region is reused by the next round
+  }
+}
+
+// Shared-memory floats the key-block split may use for its partials (0: not
+// available, every item runs whole in one warp): the operand region past the
+// attention scratch (the operand is idle during the attention phase).
+template <int B>
+__device__ __forceinline__ int att_part_floats(const DecodeParams& p, int kmax) {
+  const int act = decode_act_bytes(B, kmax);
+  const int used = decode_att_in_act(B, kmax, p.fuse_att) ? kConsumerWarps * 3 * kAttHd * 4 : 0;
+  const int kb = (p.hd <= 64) ? 32 : 16;
+  const int need = ((p.max_seq - 1) / kb + 1) * (p.hd + 2);
+  const int avail = (act - used) / 4;
+  return avail >= need ? avail : 0;
+}
+
+// Separate attention phase (large attention).
 template <int B>
 __device__ void attention_phase(const DecodeParams& p, const Smem& sm, int layer, int t,
-                                int tid_c) {
+                                int tid_c, int kmax) {
   const int warp = tid_c >> 5, lane = tid_c & 31;
-  const int items = B * p.H;
-  const int stride = p.n_ctas * kConsumerWarps;
-  const int group = p.H / p.Hkv;
-  for (int it = blockIdx.x * kConsumerWarps + warp; it < items; it += stride) {
-    const int b = it / p.H, h = it - b * p.H;
-    attend<B>(p, sm, layer, t, b, h, (h % group) == 0, false, warp, lane);
+  const int avail = att_part_floats<B>(p, kmax);
+  if (avail > 0) {
+    float* part = reinterpret_cast<float*>(
+        sm.act + (decode_att_in_act(B, kmax, p.fuse_att) ? kConsumerWarps * 3 * kAttHd * 4 : 0));
+    switch (p.hd) {
+      case 32: attention_split<B, 32>(p, sm, layer, t, tid_c, part, avail); break;
+      case 64: attention_split<B, 64>(p, sm, layer, t, tid_c, part, avail); break;
+      default: attention_split<B, 128>(p, sm, layer, t, tid_c, part, avail); break;
+    }
+  } else {
+    // items spread over all warps of all CTAs, one warp per (b, h)
+    const int items = B * p.H;
+    const int stride = p.n_ctas * kConsumerWarps;
+    const int group = p.H / p.Hkv;
+    for (int it = blockIdx.x * kConsumerWarps + warp; it < items; it += stride) {
+      const int b = it / p.H, h = it - b * p.H;
+      attend<B>(p, sm, layer, t, b, h, (h % group) == 0, false, warp, lane);
+    }
   }
   // o image -> the O phase's bulk copies; the scratch (inside the operand
   // region) -> the next bulk copy into it
@@ -1346,7 +1575,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
       if (tl && tid_c == 0) tl[0] = globaltimer();
       long long t0 = MX_CLK();
       if (kind == PH_ATT) {
-        attention_phase<B>(p, sm, layer, s, tid_c);
+        attention_phase<B>(p, sm, layer, s, tid_c, kmax);
         if (tl && tid_c == 0) tl[1] = tl[2] = globaltimer();
         const long long t1 = MX_CLK();
         c_att += t1 - t0;

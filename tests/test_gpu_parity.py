@@ -117,6 +117,29 @@ def test_results_identical_across_partition_sizes(mxlib, parts):
         assert np.array_equal(lg.view(np.uint32), outs[0][1].view(np.uint32))
 
 
+@pytest.mark.parametrize("B", [1, 8])
+def test_llama7b_width_identical_chained_vs_distributed(mxlib, parts, B):
+    """7B widths (2 layers): on 36 SMs every CTA chains the K segments of its
+    own rows; on 148 SMs the O/DOWN pieces are spread over the CTAs and
+    finished by other CTAs, and the attention runs key-block split. The row
+    sums keep the segment order either way, so tokens and logits must be
+    bit-identical; and both match the oracle."""
+    cfg = LLAMA7B.with_layers(2)
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=B))
+    prompt = prompt_tokens(40 + B, B, 5, cfg.vocab)
+    outs = []
+    for sm in (36, 148):
+        p = parts(sm, hbm=4 << 30)
+        t = mxlib.decode_task(fn, prompt, 4, want_logits=True, vocab=cfg.vocab)
+        mxlib.fn_submit(p, t)
+        assert mxlib.fn_wait(t)["status"] == 0
+        outs.append((t.tokens.copy(), t.logits.copy()))
+        mxlib.part_destroy(p)
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][1].view(np.uint32), outs[1][1].view(np.uint32))
+    _check_decode(cfg, decode_weights(cfg), prompt, 4, outs[1][0], outs[1][1])
+
+
 def test_shared_partitions_time_share_and_concurrent(mxlib):
     """N1 modes (unpartitioned streams, cooperative launches): two time-shared
     streams (148-CTA grids competing for every SM) and two concurrent ones
