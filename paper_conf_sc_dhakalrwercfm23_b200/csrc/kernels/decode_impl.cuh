@@ -1279,25 +1279,38 @@ __device__ __forceinline__ void norm_finish(const DecodeParams& p, const Smem& s
   }
 }
 
-// Operand-image phases, all consumer threads: reset the LM argmax, reduce
-// rms(x) from the producer's sums of squares over 8-row groups (the group ->
-// thread assignment depends only on kNCT, not on the grid).
+// Operand-image phases, the 4 epilogue warps only (the MMAs start as soon as
+// the operand copy lands; only the epilogue needs the RMSNorm scale): reset the
+// LM argmax, reduce rms(x) from the producer's sums of squares over 8-row
+// groups (the group -> thread assignment and the warp order are fixed: the
+// result does not depend on the grid).
 template <int B>
-__device__ __forceinline__ void prep_img(const DecodeParams& p, const Smem& sm, const Phase& ph,
-                                         int tid_c) {
-  if (ph.kind == PH_LM && tid_c < B) sm.best[tid_c] = 0ull;
+__device__ __forceinline__ void epi_prep(const DecodeParams& p, const Smem& sm, const Phase& ph,
+                                         int warp, int lane) {
+  const int q = warp & 3, et = 32 * q + lane;
+  if (ph.kind == PH_LM && et < B) sm.best[et] = 0ull;
   if (ph.kind == PH_QKV || ph.kind == PH_GU || ph.kind == PH_LM) {
     const int G8 = ph.KF >> 3;
     float acc[B];
 #pragma unroll
     for (int b = 0; b < B; ++b) acc[b] = 0.f;
-    for (int g = tid_c; g < G8; g += kNCT) {
+    for (int g = et; g < G8; g += 128) {
 #pragma unroll
       for (int b = 0; b < B; ++b) acc[b] += p.ssq[b * G8 + g];
     }
-    norm_finish<B>(p, sm, acc, ph.KF, tid_c);
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const float t = warp_sum(acc[b]);
+      if (lane == 0) sm.wsum[q * 8 + b] = t;
+    }
+    named_bar_sync(2, 128);
+    if (et < B) {
+      float t = 0.f;
+      for (int w = 0; w < 4; ++w) t += sm.wsum[w * 8 + et];
+      sm.inv[et] = 1.0f / sqrtf(t / (float)ph.KF + p.eps);
+    }
   }
-  named_bar_sync(1, kNCT);
+  named_bar_sync(2, 128);
 }
 
 __device__ __forceinline__ bool img_phase(const DecodeParams& p, int kind, int layer) {
@@ -1603,7 +1616,6 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
             __syncwarp();
           };
           if (stager && n_act > 0) copy_seg(ga);
-          prep_img<B>(p, sm, ph0, tid_c);
           if (tl && tid_c == 0) tl[1] = globaltimer();
           const long long t1 = MX_CLK();
           c_stage += t1 - t0;
@@ -1625,6 +1637,7 @@ __global__ void __launch_bounds__(kDecodeThreads, 1) decode_kernel(DecodeParams 
             }
             if (tl && lane == 0) tl[2] = globaltimer();
           } else if (warp_id >= kEpiWarp0 && warp_id < kEpiWarp0 + 4) {
+            epi_prep<B>(p, sm, ph0, warp_id, lane);
             for (int seg = ga; seg <= gb; ++seg)
               epi_dispatch<B>(p, sm, make_phase<B>(p, kind, layer, seg), k, s, warp_id, lane, tc,
                               tmem_base, w_tf);
