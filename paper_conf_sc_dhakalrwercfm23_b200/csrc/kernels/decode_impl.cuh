@@ -759,33 +759,23 @@ __device__ __forceinline__ void epi_finalize(const DecodeParams& p, const Smem& 
       u[b] = 0.f;
     }
     if (ok) {
-      // partials in segment order, two segments' loads in flight at a time
-      for (int g0 = 0; g0 < nseg; g0 += 2) {
-        float tv[2][B], tu[2][B];
+      // partials in segment order, four segments' loads (x B) in flight at a time
+      // (only O and DOWN are distributed: one value per row and sequence)
+      static_assert(!gu, "gate/up phases are never distributed");
+      constexpr int GR = 4;
+      for (int g0 = 0; g0 < nseg; g0 += GR) {
+        float tv[GR][B];
 #pragma unroll
-        for (int t = 0; t < 2; ++t) {
+        for (int t = 0; t < GR; ++t) {
 #pragma unroll
-          for (int b = 0; b < B; ++b) {
-            tv[t][b] = tu[t][b] = 0.f;
-            if (g0 + t < nseg) {
-              if (gu) {
-                const float2 x2 = __ldcg(reinterpret_cast<const float2*>(kpart_at(p, ph0, g0 + t, b, 2 * row)));
-                tv[t][b] = x2.x;
-                tu[t][b] = x2.y;
-              } else {
-                tv[t][b] = __ldcg(kpart_at(p, ph0, g0 + t, b, row));
-              }
-            }
-          }
+          for (int b = 0; b < B; ++b)
+            tv[t][b] = (g0 + t < nseg) ? __ldcg(kpart_at(p, ph0, g0 + t, b, row)) : 0.f;
         }
 #pragma unroll
-        for (int t = 0; t < 2; ++t) {
+        for (int t = 0; t < GR; ++t) {
           if (g0 + t < nseg) {
 #pragma unroll
-            for (int b = 0; b < B; ++b) {
-              v[b] = (g0 + t == 0) ? tv[t][b] : tv[t][b] + v[b];
-              u[b] = (g0 + t == 0) ? tu[t][b] : tu[t][b] + u[b];
-            }
+            for (int b = 0; b < B; ++b) v[b] = (g0 + t == 0) ? tv[t][b] : tv[t][b] + v[b];
           }
         }
       }
