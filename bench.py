@@ -400,11 +400,16 @@ def decode_traffic():
 
 
 def kernel_source_hash():
+    """sha256 of the decode kernel's code (decode_impl.cuh + common.cuh) with
+    comments and blank lines removed, so documentation edits keep the stamp."""
     import hashlib
+    import re
     h = hashlib.sha256()
     for f in ("decode_impl.cuh", "common.cuh"):
-        with open(os.path.join(ROOT, "paper_conf_sc_dhakalrwercfm23_b200", "csrc", "kernels", f), "rb") as fh:
-            h.update(fh.read())
+        with open(os.path.join(ROOT, "paper_conf_sc_dhakalrwercfm23_b200", "csrc", "kernels", f)) as fh:
+            src = re.sub(r"/\*.*?\*/", "", fh.read(), flags=re.S)
+        lines = (re.sub(r"//.*$", "", ln).rstrip() for ln in src.splitlines())
+        h.update("\n".join(ln for ln in lines if ln).encode())
     return h.hexdigest()
 
 

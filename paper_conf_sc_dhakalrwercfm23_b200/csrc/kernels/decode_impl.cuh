@@ -24,17 +24,25 @@
 //    epilogue warps drain the accumulators (tcgen05.ld) and apply the phase's
 //    epilogue (residual add, SiLU-gate, argmax). The CUDA cores no longer touch
 //    the weights, so the kernel is HBM-bound at any clock.
-//  * weights (>98% of the bytes) are streamed by a producer thread with 3-D
-//    tiled TMA (one CUtensorMap per matrix kind covering all layers) into a
-//    ring of 16 KiB stages ([128 rows][64 columns] bf16, K-major SWIZZLE_128B:
-//    exactly the UMMA operand layout) guarded by mbarriers; MMA completion
-//    (tcgen05.commit) frees a stage. The weight stream is static, so the
-//    producer runs ahead ACROSS phase barriers.
-//  * rows are split across CTAs in multiples of 8 with a per-phase rotation;
-//    a CTA's rows are covered by 128-row boxes plus 32- and 8-row boxes for
-//    its tail (rows of other CTAs are never read). Every output row is owned
-//    by exactly one CTA and its K reduction order is fixed, so results do not
-//    depend on the partition size.
+//  * weights (>98% of the bytes) are streamed by a producer thread with 4-D
+//    tiled TMA (one CUtensorMap per matrix kind and box height, covering all
+//    layers) into a ring of 32 KiB stages (a tile's exact rows x up to 8
+//    64-column blocks, K-major SWIZZLE_128B: the UMMA A-operand layout)
+//    guarded by mbarriers; MMA completion (tcgen05.commit) frees a stage. The
+//    weight stream is static, so the producer runs ahead ACROSS phase barriers.
+//  * rows are split across CTAs in multiples of 8 with a per-phase rotation
+//    (rows of other CTAs are never read); inputs wider than the operand
+//    region run as K segments whose partials the row owner chains in segment
+//    order. When that split would leave < 64 rows per CTA (O/DOWN of a 7B on
+//    148 SMs) the (segment, 8-row group) pieces are spread over the CTAs and
+//    statically assigned CTAs finish each 128-row block from the partials,
+//    summed in the same segment order. Segment boundaries depend only on the
+//    shape, so results do not depend on the partition size.
+//  * the phase inputs are operand images written by the producing epilogue
+//    (one bulk copy per K segment); the RMSNorm scale is an output-column
+//    factor the epilogue warps reduce while the MMAs run.
+//  * a separate attention phase splits each (sequence, head) over warps by
+//    key block (block partials folded in block order, flash-decoding style).
 #include <cfloat>
 
 #include "common.cuh"
