@@ -117,8 +117,8 @@ def test_results_identical_across_partition_sizes(mxlib, parts):
         assert np.array_equal(lg.view(np.uint32), outs[0][1].view(np.uint32))
 
 
-@pytest.mark.parametrize("B", [1, 8])
-def test_llama7b_width_identical_chained_vs_distributed(mxlib, parts, B):
+@pytest.mark.parametrize("B,sms", [(1, (36, 148)), (8, (36, 148)), (3, (52, 100))])
+def test_llama7b_width_identical_chained_vs_distributed(mxlib, parts, B, sms):
     """7B widths (2 layers): on 36 SMs every CTA chains the K segments of its
     own rows; on 148 SMs the O/DOWN pieces are spread over the CTAs and
     finished by other CTAs, and the attention runs key-block split. The row
@@ -128,7 +128,7 @@ def test_llama7b_width_identical_chained_vs_distributed(mxlib, parts, B):
     fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=B))
     prompt = prompt_tokens(40 + B, B, 5, cfg.vocab)
     outs = []
-    for sm in (36, 148):
+    for sm in sms:
         p = parts(sm, hbm=4 << 30)
         t = mxlib.decode_task(fn, prompt, 4, want_logits=True, vocab=cfg.vocab)
         mxlib.fn_submit(p, t)

@@ -126,11 +126,15 @@ def test_c3_llama7b_all_32_layers(mxlib, parts):
     print(f"7B L32 B=1 on 148 SMs: tokens identical, max logit rel {rel:.2e}")
 
 
-@pytest.mark.parametrize("cfg,B,P,sm", [(TINY, 1, 8, 8), (RAGGED, 2, 300, 12), (TINY, 4, 500, 16)])
+@pytest.mark.parametrize("cfg,B,P,sm", [(TINY, 1, 8, 8), (RAGGED, 2, 300, 12), (TINY, 4, 500, 16),
+                                         (TINY, 8, 500, 16), (replace(TINY, n_heads=2, n_kv_heads=2, head_dim=128), 8, 480, 20)])
 def test_longest_context_max_seq_512(mxlib, parts, cfg, B, P, sm):
     """P + G - 1 = max_seq = 512 (the ABI's cap, kMaxSeqCap: 16 attention scores
-    per lane): the last steps attend over all 512 cached positions. CUDA-core
-    GEMV at B = 1-2 (GQA 6/2, hd 32 for RAGGED), tensor-core GEMV at B = 4."""
+    per lane): the last steps attend over all 512 cached positions. GQA 6/2 hd 32
+    (RAGGED), fused attention at B <= 4; at B = 8 a separate attention phase
+    with the key-block split (hd 64: 32-key blocks throughout; hd 128: 16-key
+    blocks while their partials fit the operand region, t < 208 here, then one
+    warp per head)."""
     cfg = replace(cfg, max_seq=512)
     G = 513 - P
     p = parts(sm)
