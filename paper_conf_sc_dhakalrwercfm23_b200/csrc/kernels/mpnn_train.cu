@@ -50,8 +50,8 @@ constexpr int kOffRed = kOffOff4 + kA * 5 * 4;      // float [4][kF] column part
 constexpr int kOffVec = kOffRed + 4 * kF * 4;       // float [4][kF]: r, a, da, dr
 constexpr int kOffC = kOffVec + 4 * kF * 4;         // float [kF] bias c
 constexpr int kOffMisc = kOffC + kF * 4;            // float [16]
-constexpr int kOffBar = kOffMisc + 64;              // uint64 MMA-done mbarrier
-constexpr int kOffTmem = kOffBar + 8;               // uint32 TMEM base
+constexpr int kOffBar = kOffMisc + 64;              // uint64 MMA-done mbarrier, uint64 copy-done mbarrier
+constexpr int kOffTmem = kOffBar + 16;              // uint32 TMEM base
 constexpr int kTrainSmem = kOffTmem + 8 + 1024;     // + alignment slack
 // setup-only aliases inside Op1 (before the first gather)
 constexpr int kOffEdges = kOffOp1;                  // int4 [kTE]
@@ -139,10 +139,20 @@ __device__ void gather(uint8_t* out_hi, uint8_t* out_lo, const uint8_t* src_hi, 
   }
 }
 
-// Copy a precomputed operand image (global, L2-resident) into shared memory.
-__device__ __forceinline__ void copy_img(uint8_t* dst, const uint8_t* __restrict__ src, int bytes, int tid) {
-  for (int i = tid * 16; i < bytes; i += kThreads * 16)
-    *reinterpret_cast<uint4*>(dst + i) = *reinterpret_cast<const uint4*>(src + i);
+// Copy a precomputed operand image (global, L2-resident) into shared memory:
+// one bulk (async-proxy) copy issued by ONE thread, completing on
+// `cbar`; the other threads go on (neighbour gathers) while it lands. The
+// destination's previous readers (MMAs) have completed (waited + barrier).
+__device__ __forceinline__ void copy_img_async(uint8_t* dst, const uint8_t* src, int bytes,
+                                               uint64_t* cbar) {
+  fence_proxy_async();   // earlier generic writes of this shared memory -> async-proxy writes
+  mbar_arrive_expect_tx(cbar, (uint32_t)bytes);
+  for (int o = 0; o < bytes; o += 16384) bulk_g2s(dst + o, src + o, (uint32_t)min(16384, bytes - o), cbar);
+}
+__device__ __forceinline__ void copy_wait(uint64_t* cbar, uint32_t& cph) {
+  while (!mbar_try_wait(cbar, cph)) {
+  }
+  cph ^= 1u;
 }
 // per matrix (U, W_0..W_3): forward image hi | lo ([f][k]) and backward image ([k][f], hi)
 constexpr int kImgBytes = 3 * kOp;
@@ -225,8 +235,10 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   const float* c1 = p.params + p.off[8];
   const float* w2 = p.params + p.off[9];
   const float c2 = p.params[p.off[10]];
+  uint64_t* cbar = bar + 1;
   if (tid == 0) {
     mbar_init(bar, 1);
+    mbar_init(cbar, 1);
     fence_mbar_init();
   }
   if (warp == 0) tmem_alloc(tmem_slot, kTmemCols);
@@ -236,7 +248,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   tc_fence_after();
   const uint32_t tmem = __shfl_sync(0xffffffffu, *tmem_slot, 0);
   const uint32_t bar_s = smem_u32(bar);
-  uint32_t ph = 0;
+  uint32_t ph = 0, cph = 0;   // MMA-done / copy-done mbarrier parities (every thread tracks both)
   const uint32_t s0 = smem_u32(op0), s1 = smem_u32(op1), s2 = smem_u32(op2);
   const uint32_t acc0 = tmem, acc1 = tmem + 128u;
   // this thread's TMEM row (lane) and column half
@@ -356,11 +368,12 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         if (b >= 0 && !(present & (1 << b))) continue;
         // operands: A = H (b = -1) or S_b, B = U or W_b, both hi/lo (3 products)
         __syncthreads();   // previous MMAs done (waited) -> S / W buffers free
+        if (tid == 0) copy_img_async(op2, p.wimg + (size_t)(b + 1) * kImgBytes, 2 * kOp, cbar);   // W (hi | lo)
         if (b >= 0) gather(op1, op1 + kOp, op0, op0 + kOp, off4, nbr, na, b, false, tid);
-        copy_img(op2, p.wimg + (size_t)(b + 1) * kImgBytes, 2 * kOp, tid);   // W (hi | lo)
         fence_proxy_async();
         tc_fence_before();
         __syncthreads();
+        if (warp == 0) copy_wait(cbar, cph); else cph ^= 1u;
         if (warp == 0) {
           tc_fence_after();
           const uint32_t a = b < 0 ? s0 : s1;
@@ -460,6 +473,9 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
     uint8_t* hv = op2 + kOp;       // [v][k]  (gather source for s_b)
     const uint32_t sdqT = s0, sdq = s0 + kOp, shT = s1, sX = s1 + kOp, sWt = s2;
     for (int t = p.T - 1; t >= 0; --t) {
+      // U^T into Wt while (a) and (b) run (Wt's last readers, the previous
+      // step's MMAs, were waited; (b) writes only the other half, hv)
+      if (tid == 0) copy_img_async(Wt, p.wimg + 2 * kOp, kOp, cbar);
       // (a) dq from dh (acc1, or the readout's dr at the last step) and the mask
       {
         float dh64[64];
@@ -505,11 +521,11 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
             *reinterpret_cast<uint16_t*>(hv + elem_off(8 * ch + j, k)) = f32_to_bf16_rne(f[j]);
         }
       }
-      copy_img(Wt, p.wimg + 2 * kOp, kOp, tid);                     // U^T
       fence_proxy_async();
       tc_fence_before();
       __syncthreads();
       if (tid < F) G[p.off[6] + tid] += (red[tid] + red[F + tid]) + (red[2 * F + tid] + red[3 * F + tid]);   // dc
+      if (warp == 0) copy_wait(cbar, cph); else cph ^= 1u;   // U^T (issued at the step start)
       if (warp == 0) {
         tc_fence_after();
         mma_128(acc0, shT, sdqT, false);     // dU^T[k][f] = sum_v h[v][k] dq[v][f]
@@ -549,11 +565,12 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         flush(G + p.off[1] + (size_t)b * F * F, t == p.T - 1);      // dW_b
         tc_fence_before();
         __syncthreads();   // X and Wt free
+        if (tid == 0) copy_img_async(Wt, p.wimg + (size_t)(b + 1) * kImgBytes + 2 * kOp, kOp, cbar);   // W_b^T
         gather(X, nullptr, dq, nullptr, off4, nbr, na, b, false, tid);  // gq_b [v][f]
-        copy_img(Wt, p.wimg + (size_t)(b + 1) * kImgBytes + 2 * kOp, kOp, tid);   // W_b^T
         fence_proxy_async();
         tc_fence_before();
         __syncthreads();
+        if (warp == 0) copy_wait(cbar, cph); else cph ^= 1u;
         if (warp == 0) {
           tc_fence_after();
           mma_128(acc1, sX, sWt, true);      // dh[v][k] += sum_f gq_b[v][f] W_b[f][k]
