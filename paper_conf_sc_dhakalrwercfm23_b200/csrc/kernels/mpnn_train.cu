@@ -217,9 +217,6 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   int* nbr = reinterpret_cast<int*>(sm + kOffNbr);
   int* off4 = reinterpret_cast<int*>(sm + kOffOff4);
   float* red = reinterpret_cast<float*>(sm + kOffRed);
-  float* rr = reinterpret_cast<float*>(sm + kOffVec);
-  float* aa = rr + kF;
-  float* da = aa + kF;
   float* cvec = reinterpret_cast<float*>(sm + kOffC);
   float* misc = reinterpret_cast<float*>(sm + kOffMisc);
   uint64_t* bar = reinterpret_cast<uint64_t*>(sm + kOffBar);
@@ -407,52 +404,91 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       }
     }
     __syncthreads();
-    // ===================== readout, loss, head gradients (per molecule) ==========
-    const float* hT = hs + (size_t)p.T * F * kA;
-    for (int m = m0; m < m1; ++m) {
-      const int ab = p.atom_off[m] - a0, ae = p.atom_off[m + 1] - a0;
-      if (tid < F) {
+    // ===================== readout, loss, head gradients (all molecules of the tile) ==
+    // Batched over the tile's molecules (the per-molecule version left half the
+    // threads idle and paid a global round trip per molecule and step); every
+    // sum keeps the per-molecule version's order, so the results are unchanged.
+    // Scratch: the three operand buffers (64 KiB each) are free until the
+    // backward stages its first operands (h^T comes from the saved fp32 rows).
+    {
+      const float* hT = hs + (size_t)p.T * F * kA;
+      const int nm = m1 - m0;                             // <= kA (every molecule has an atom)
+      float* Rs = reinterpret_cast<float*>(op0);          // [nm][F] r_m (readout sums)
+      float* As = reinterpret_cast<float*>(op1);          // [nm][F] a_m (pre-activation)
+      float* Ds = reinterpret_cast<float*>(op2);          // [nm][F] da_m
+      float* Ys = red;                                    // [nm] dy_m (red: [4][kF] floats)
+      const int f = tid & (kF - 1), half = tid >> 7;     // two molecule halves in parallel
+      // r_m[k] = sum over m's atoms (atom order) of h^T[k][v]
+      for (int m = half; m < nm; m += 2) {
+        const int ab = p.atom_off[m0 + m] - a0, ae = p.atom_off[m0 + m + 1] - a0;
         float r = 0.f;
-        for (int v = ab; v < ae; ++v) r += hT[tid * kA + v];
-        rr[tid] = r;
+        for (int v = ab; v < ae; ++v) r += hT[f * kA + v];
+        Rs[m * F + f] = r;
       }
       __syncthreads();
-      if (tid < F) {
-        float a = c1[tid];
-        for (int k = 0; k < F; ++k) a = fmaf(W1[tid * F + k], rr[k], a);
-        aa[tid] = a;
+      // a_m[f] = c1[f] + sum_k W1[f][k] r_m[k] (k order), 8 molecules per pass
+      for (int mb = 8 * half; mb < nm; mb += 16) {
+        float acc[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = c1[f];
+        for (int k = 0; k < F; ++k) {
+          const float w = W1[f * F + k];
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            if (mb + i < nm) acc[i] = fmaf(w, Rs[(mb + i) * F + k], acc[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          if (mb + i < nm) As[(mb + i) * F + f] = acc[i];
       }
       __syncthreads();
-      if (warp == 0) {
+      // y_m = c2 + w2 . relu(a_m) (lane-strided partials + the fixed shuffle tree), dy_m
+      for (int m = warp; m < nm; m += kThreads / 32) {
         float part = 0.f;
-        for (int f = lane; f < F; f += 32) part = fmaf(w2[f], fmaxf(aa[f], 0.f), part);
+        for (int ff = lane; ff < F; ff += 32) part = fmaf(w2[ff], fmaxf(As[m * F + ff], 0.f), part);
         part = warp_sum(part);
         if (lane == 0) {
           const float y = part + c2;
-          p.y[m] = y;
-          p.out[m] = y;
-          misc[0] = 2.0f * (y - p.targets[m]) / (float)p.n_mol;   // dy
+          p.y[m0 + m] = y;
+          p.out[m0 + m] = y;
+          Ys[m] = 2.0f * (y - p.targets[m0 + m]) / (float)p.n_mol;   // dy
         }
       }
       __syncthreads();
-      const float dy = misc[0];
+      // da_m[f]; head gradients summed in molecule order (as the per-molecule RMWs)
       if (tid < F) {
-        G[p.off[9] + tid] += dy * fmaxf(aa[tid], 0.f);              // dw2
-        const float d = (aa[tid] > 0.f) ? dy * w2[tid] : 0.f;        // da
-        da[tid] = d;
-        G[p.off[8] + tid] += d;                                      // dc1
-      }
-      if (tid == 0) G[p.off[10]] += dy;                              // dc2
-      if (tid < F) {
-        rm[(m - m0) * F + tid] = rr[tid];
-        dam[(m - m0) * F + tid] = da[tid];
+        float gw2 = G[p.off[9] + f], gc1 = G[p.off[8] + f], gc2 = (f == 0) ? G[p.off[10]] : 0.f;
+        for (int m = 0; m < nm; ++m) {
+          const float dy = Ys[m], a = As[m * F + f];
+          gw2 += dy * fmaxf(a, 0.f);
+          const float d = (a > 0.f) ? dy * w2[f] : 0.f;
+          Ds[m * F + f] = d;
+          gc1 += d;
+          if (f == 0) gc2 += dy;
+          rm[m * F + f] = Rs[m * F + f];
+          dam[m * F + f] = d;
+        }
+        G[p.off[9] + f] = gw2;
+        G[p.off[8] + f] = gc1;
+        if (f == 0) G[p.off[10]] = gc2;
       }
       __syncthreads();
-      if (tid < F) {
-        float s = 0.f;
-        for (int f = 0; f < F; ++f) s = fmaf(W1[f * F + tid], da[f], s);
-        drm[(m - m0) * F + tid] = s;                                 // dr: dh^T of every atom of m
+      // dr_m[k] = sum_f W1[f][k] da_m[f] (f order): dh^T of every atom of m
+      for (int mb = 8 * half; mb < nm; mb += 16) {
+        float acc[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) acc[i] = 0.f;
+        for (int ff = 0; ff < F; ++ff) {
+          const float w = W1[ff * F + f];
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            if (mb + i < nm) acc[i] = fmaf(w, Ds[(mb + i) * F + ff], acc[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          if (mb + i < nm) drm[(mb + i) * F + f] = acc[i];
       }
+      fence_proxy_async();   // generic scratch writes before the backward's async-proxy copies / MMAs
       __syncthreads();
     }
     // dW1 += sum_m da_m r_m^T (molecule order, one pass over the partial)
