@@ -255,10 +255,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   for (int tile = blockIdx.x; tile < p.n_tiles; tile += p.n_ctas) {
     float* G = p.partials + (uint64_t)tile * p.n_params;
     float* hs = p.hsave + (uint64_t)tile * (p.T + 5) * kF * kA;   // [T+1][k][v]
-    float* dh0 = hs + (uint64_t)(p.T + 1) * kF * kA;               // [k][v]
-    float* drm = dh0 + (uint64_t)kF * kA;                          // [molecule][k]
-    float* rm = drm + (uint64_t)kF * kA;                           // [molecule][k]
-    float* dam = rm + (uint64_t)kF * kA;                           // [molecule][f]
+    float* drm = hs + (uint64_t)(p.T + 2) * kF * kA;               // [molecule][k]
     const int m0 = p.tile_off[tile], m1 = p.tile_off[tile + 1];
     const int a0 = p.atom_off[m0], na = p.atom_off[m1] - a0;
     const int e0 = p.edge_off[m0], ne = p.edge_off[m1] - e0;
@@ -465,14 +462,19 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
           Ds[m * F + f] = d;
           gc1 += d;
           if (f == 0) gc2 += dy;
-          rm[m * F + f] = Rs[m * F + f];
-          dam[m * F + f] = d;
         }
         G[p.off[9] + f] = gw2;
         G[p.off[8] + f] = gc1;
         if (f == 0) G[p.off[10]] = gc2;
       }
       __syncthreads();
+      // dW1 += sum_m da_m r_m^T (molecule order, one pass over the partial)
+      for (int i = tid; i < F * F; i += kThreads) {
+        const int fi = i / F, k = i - fi * F;
+        float g = 0.f;
+        for (int m = 0; m < nm; ++m) g = fmaf(Ds[m * F + fi], Rs[m * F + k], g);
+        G[p.off[7] + i] += g;
+      }
       // dr_m[k] = sum_f W1[f][k] da_m[f] (f order): dh^T of every atom of m
       for (int mb = 8 * half; mb < nm; mb += 16) {
         float acc[8];
@@ -490,13 +492,6 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       }
       fence_proxy_async();   // generic scratch writes before the backward's async-proxy copies / MMAs
       __syncthreads();
-    }
-    // dW1 += sum_m da_m r_m^T (molecule order, one pass over the partial)
-    for (int i = tid; i < F * F; i += kThreads) {
-      const int f = i / F, k = i - f * F;
-      float g = 0.f;
-      for (int m = 0; m < m1 - m0; ++m) g = fmaf(dam[m * F + f], rm[m * F + k], g);
-      G[p.off[7] + i] += g;
     }
     // ===================== backward through the T message-passing steps ==========
     // per step (reverse): dq = dh * [h^{t+1} > 0]; dc += sum_v dq; dU += dq^T h;
@@ -617,17 +612,26 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       tc_fence_before();
       __syncthreads();
     }
-    // dE[type_v] += dh^0_v (atom order): dh^0 ([k][v], fp32) through the scratch
+    // dE[type_v] += dh^0_v (atom order): dh^0 through shared memory ([v][k], row
+    // stride F + 1: conflict-free both ways), per-type sums in shared memory
+    // (zero-initialised like the partial, so the sums are the same bits)
     {
+      float* Hs = reinterpret_cast<float*>(op0);   // [kA][F + 1] (op0 + op1)
+      float* Es = reinterpret_cast<float*>(op2);   // [n_types][F]
+      const int n_types = (int)(p.off[1] - p.off[0]) / F;   // E is [n_types][F], W_0 follows
       float dh64[64];
       tmem_row64(acc1 + lane_off + (uint32_t)tc0, dh64);
       const int v = trow;
 #pragma unroll
-      for (int j = 0; j < 64; ++j) dh0[(tc0 + j) * kA + v] = (v < na) ? dh64[j] : 0.f;
+      for (int j = 0; j < 64; ++j) Hs[v * (F + 1) + tc0 + j] = (v < na) ? dh64[j] : 0.f;
+      for (int i = tid; i < n_types * F; i += kThreads) Es[i] = 0.f;
+      __syncthreads();
+      if (tid < F)
+        for (int vv = 0; vv < na; ++vv) Es[(int)p.atom_type[a0 + vv] * F + tid] += Hs[vv * (F + 1) + tid];
+      __syncthreads();
+      for (int i = tid; i < n_types * F; i += kThreads) G[p.off[0] + i] += Es[i];
     }
-    __syncthreads();
-    if (tid < F)
-      for (int v = 0; v < na; ++v) G[p.off[0] + (int)p.atom_type[a0 + v] * F + tid] += dh0[tid * kA + v];
+    fence_proxy_async();   // generic scratch writes before the next tile's async-proxy copies
     tc_fence_before();
     __syncthreads();
   }
