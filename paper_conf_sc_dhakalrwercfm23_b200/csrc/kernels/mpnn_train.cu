@@ -262,11 +262,10 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
     {
       // zero this tile's partial except U and the W_b the backward writes whole
       // (W_b of bond types absent from the tile stay zero)
-      for (int i = tid; i < p.n_params; i += kThreads) {
-        const bool u_or_w = (i >= (int)p.off[1] && i < (int)p.off[1] + 4 * F * F) ||
-                            (i >= (int)p.off[5] && i < (int)p.off[5] + F * F);
-        if (!u_or_w) G[i] = 0.f;
-      }
+      // (layout: E, W_0..W_3, U, c, W1, c1, w2, c2 in offset order; the zeroed
+      // ranges [0, off[1]) and [off[6], n_params) are everything but W_b and U)
+      for (int i = tid; i < (int)p.off[1]; i += kThreads) G[i] = 0.f;
+      for (int i = (int)p.off[6] + tid; i < p.n_params; i += kThreads) G[i] = 0.f;
     }
     // --- tile CSR (as the inference kernel): edges in tile-local atom ids --------
     for (int i = tid; i < kA; i += kThreads) mol_e[i] = make_int2(0, 0);
@@ -624,12 +623,21 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
       const int v = trow;
 #pragma unroll
       for (int j = 0; j < 64; ++j) Hs[v * (F + 1) + tc0 + j] = (v < na) ? dh64[j] : 0.f;
-      for (int i = tid; i < n_types * F; i += kThreads) Es[i] = 0.f;
-      __syncthreads();
-      if (tid < F)
-        for (int vv = 0; vv < na; ++vv) Es[(int)p.atom_type[a0 + vv] * F + tid] += Hs[vv * (F + 1) + tid];
-      __syncthreads();
-      for (int i = tid; i < n_types * F; i += kThreads) G[p.off[0] + i] += Es[i];
+      if (n_types * F * 4 <= 2 * kOp) {
+        for (int i = tid; i < n_types * F; i += kThreads) Es[i] = 0.f;
+        __syncthreads();
+        if (tid < F)
+          for (int vv = 0; vv < na; ++vv) Es[(int)p.atom_type[a0 + vv] * F + tid] += Hs[vv * (F + 1) + tid];
+        __syncthreads();
+        for (int i = tid; i < n_types * F; i += kThreads) G[p.off[0] + i] += Es[i];
+      } else {
+        // more than 128 atom types: the per-type sums do not fit op2; accumulate
+        // in the (zeroed) partial directly, same order
+        __syncthreads();
+        if (tid < F)
+          for (int vv = 0; vv < na; ++vv)
+            G[p.off[0] + (int)p.atom_type[a0 + vv] * F + tid] += Hs[vv * (F + 1) + tid];
+      }
     }
     fence_proxy_async();   // generic scratch writes before the next tile's async-proxy copies
     tc_fence_before();

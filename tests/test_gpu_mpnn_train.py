@@ -108,3 +108,25 @@ def test_train_rejects_shared_weights_and_missing_targets(mxlib, parts):
     with pytest.raises(mxlib.MxError) as e:
         mxlib.fn_submit(p, t)
     assert e.value.code == mxlib.MX_EINVAL
+
+
+def test_train_step_parity_many_atom_types(mxlib, parts):
+    """200 atom types: the embedding gradient's per-type sums no longer fit the
+    shared-memory scratch and are accumulated in the tile partial directly
+    (same order); still within the update tolerance of the oracle."""
+    from dataclasses import replace
+    cfg = replace(MPNN, n_atom_types=200)
+    p = parts(8, hbm=512 << 20)
+    M = 32
+    fn = mxlib.fn_register(mxlib.mpnn_train_desc(cfg, M, M * 32, M * 64))
+    mxlib.fn_load(fn, p)
+    w0 = mpnn_weights(cfg)
+    mol, tg, lr = molecules(23, M), ip_targets(23, M), 0.5
+    t = mxlib.mpnn_train_task(fn, mol, tg, lr)
+    mxlib.fn_submit(p, t)
+    assert mxlib.fn_wait(t)["status"] == 0
+    new_o, loss_o, ys_o, _ = ot.train_step(w0, mol, tg, cfg.steps, lr)
+    assert np.max(np.abs(t.ip - ys_o)) / np.max(np.abs(ys_o)) <= TOL
+    assert abs(float(t.loss[0]) - loss_o) / loss_o <= TOL
+    _check_update(w0, _read(mxlib, fn, p, w0), new_o)
+
