@@ -220,6 +220,27 @@ def test_split_k_batch8_ragged_segments(mxlib, parts):
         print(f"split-K B={B}: max rel err {rel:.2e}")
 
 
+def test_split_k_chained_vs_distributed_small(mxlib, parts):
+    """The distributed DOWN phase (3 K segments, d = 2056 rows < 64 x 40 CTAs)
+    and the key-block split attention at a size compute-sanitizer can afford:
+    20 SMs (chained) vs 40 SMs (distributed) give bit-identical outputs, and
+    both match the oracle."""
+    cfg = SPLITK
+    fn = mxlib.fn_register(mxlib.decode_desc(cfg, max_batch=8))
+    prompt = prompt_tokens(77, 8, 5, cfg.vocab)
+    outs = []
+    for sm in (20, 40):
+        p = parts(sm, hbm=1 << 30)
+        t = mxlib.decode_task(fn, prompt, 4, want_logits=True, vocab=cfg.vocab)
+        mxlib.fn_submit(p, t)
+        assert mxlib.fn_wait(t)["status"] == 0
+        outs.append((t.tokens.copy(), t.logits.copy()))
+        mxlib.part_destroy(p)
+    assert np.array_equal(outs[0][0], outs[1][0])
+    assert np.array_equal(outs[0][1].view(np.uint32), outs[1][1].view(np.uint32))
+    _check_decode(cfg, decode_weights(cfg), prompt, 4, outs[1][0], outs[1][1])
+
+
 def test_c3_llama7b_width_batch8(mxlib, parts):
     """configs[2] widths at batch 8 (every phase but O runs split-K), 2 layers."""
     cfg = LLAMA7B.with_layers(2)
