@@ -52,7 +52,11 @@ constexpr int kOffC = kOffVec + 4 * kF * 4;         // float [kF] bias c
 constexpr int kOffMisc = kOffC + kF * 4;            // float [16]
 constexpr int kOffBar = kOffMisc + 64;              // uint64 MMA-done mbarrier, uint64 copy-done mbarrier
 constexpr int kOffTmem = kOffBar + 16;              // uint32 TMEM base
-constexpr int kTrainSmem = kOffTmem + 8 + 1024;     // + alignment slack
+constexpr int kMaskT = 8;                            // steps whose ReLU masks fit shared memory
+constexpr int kMaskW = 5;                            // words per row (4 + 1 pad: conflict-free)
+constexpr int kOffMask = kOffTmem + 16;              // uint32 [kMaskT][kA][kMaskW]: bit f of row v = h^{t+1}[v][f] > 0
+constexpr int kTrainSmem = kOffMask + kMaskT * kA * kMaskW * 4 + 1024;   // + alignment slack
+static_assert(kTrainSmem <= 227 * 1024, "shared memory plan");
 // setup-only aliases inside Op1 (before the first gather)
 constexpr int kOffEdges = kOffOp1;                  // int4 [kTE]
 constexpr int kOffMolE = kOffOp1 + 16 * kTE;        // int2 [kA]
@@ -221,6 +225,8 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
   float* misc = reinterpret_cast<float*>(sm + kOffMisc);
   uint64_t* bar = reinterpret_cast<uint64_t*>(sm + kOffBar);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sm + kOffTmem);
+  uint32_t* rmask = reinterpret_cast<uint32_t*>(sm + kOffMask);
+  const bool masks_smem = p.T <= kMaskT;   // else the backward reads h^{t+1} from the saved rows
   int4* ed = reinterpret_cast<int4*>(sm + kOffEdges);
   int2* mol_e = reinterpret_cast<int2*>(sm + kOffMolE);
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -386,6 +392,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         __syncthreads();   // every warp read its accumulator rows before H is overwritten
         const int v = trow;
         float* hn = hs + (size_t)(t + 1) * F * kA;
+        uint32_t bits[2] = {0u, 0u};
 #pragma unroll
         for (int c8 = 0; c8 < 8; ++c8) {
           float o[8];
@@ -394,8 +401,14 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
             const int f = tc0 + 8 * c8 + j;
             o[j] = (v < na) ? fmaxf(v64[8 * c8 + j] + cvec[f], 0.f) : 0.f;
             hn[f * kA + v] = o[j];
+            bits[c8 >> 2] |= (o[j] > 0.f ? 1u : 0u) << ((8 * c8 + j) & 31);
           }
           put8(op0, op0 + kOp, v, (tc0 >> 3) + c8, o);
+        }
+        if (masks_smem) {
+          uint32_t* mrow = rmask + ((size_t)t * kA + v) * kMaskW + (tc0 >> 5);
+          mrow[0] = bits[0];
+          mrow[1] = bits[1];
         }
       }
     }
@@ -521,14 +534,25 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         tc_fence_before();
         __syncthreads();   // acc1 read everywhere; operands of step t+1 free
         const float* hn = hs + (size_t)(t + 1) * F * kA;
+        uint32_t mb[2] = {0u, 0u};   // ReLU mask bits of h^{t+1}, this thread's row and 64 columns
+        if (masks_smem) {
+          const uint32_t* mrow = rmask + ((size_t)t * kA + v) * kMaskW + (tc0 >> 5);
+          mb[0] = mrow[0];
+          mb[1] = mrow[1];
+        }
 #pragma unroll
         for (int c8 = 0; c8 < 8; ++c8) {
           float o[8];
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             const int f = tc0 + 8 * c8 + j;
-            o[j] = (v < na && hn[f * kA + v] > 0.f) ? dh64[8 * c8 + j] : 0.f;
-            *reinterpret_cast<uint16_t*>(dqT + elem_off(f, v)) = f32_to_bf16_rne(o[j]);
+            const bool pos = masks_smem ? ((mb[c8 >> 2] >> ((8 * c8 + j) & 31)) & 1u) != 0u
+                                        : (v < na && hn[f * kA + v] > 0.f);
+            o[j] = pos ? dh64[8 * c8 + j] : 0.f;
+            // dqT[f][v]: lanes v, v + 1 (v even) share one 32-bit word
+            const uint32_t bq = f32_to_bf16_rne(o[j]);
+            const uint32_t bn = __shfl_down_sync(0xffffffffu, bq, 1);
+            if ((lane & 1) == 0) *reinterpret_cast<uint32_t*>(dqT + elem_off(f, v)) = bq | (bn << 16);
             // dc: column sums over this warp's 32 rows (fixed shuffle tree)
             const float cs = warp_sum(o[j]);
             if (lane == 0) red[(warp & 3) * F + f] = cs;
