@@ -130,3 +130,23 @@ def test_train_step_parity_many_atom_types(mxlib, parts):
     assert abs(float(t.loss[0]) - loss_o) / loss_o <= TOL
     _check_update(w0, _read(mxlib, fn, p, w0), new_o)
 
+
+
+def test_train_step_parity_nine_steps(mxlib, parts):
+    """T = 9 message-passing steps: more ReLU masks than the shared-memory bit
+    store holds (8), so the backward reads h^{t+1} from the saved fp32 rows."""
+    from dataclasses import replace
+    cfg = replace(MPNN, steps=9)
+    p = parts(4, hbm=512 << 20)
+    M = 16
+    fn = mxlib.fn_register(mxlib.mpnn_train_desc(cfg, M, M * 32, M * 64))
+    mxlib.fn_load(fn, p)
+    w0 = mpnn_weights(cfg)
+    mol, tg, lr = molecules(25, M), ip_targets(25, M), 0.5
+    t = mxlib.mpnn_train_task(fn, mol, tg, lr)
+    mxlib.fn_submit(p, t)
+    assert mxlib.fn_wait(t)["status"] == 0
+    new_o, loss_o, ys_o, _ = ot.train_step(w0, mol, tg, cfg.steps, lr)
+    assert np.max(np.abs(t.ip - ys_o)) / np.max(np.abs(ys_o)) <= TOL
+    assert abs(float(t.loss[0]) - loss_o) / loss_o <= TOL
+    _check_update(w0, _read(mxlib, fn, p, w0), new_o)
