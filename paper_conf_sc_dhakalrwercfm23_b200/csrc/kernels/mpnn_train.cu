@@ -75,17 +75,22 @@ __device__ __forceinline__ uint4 pack8(const uint16_t (&v)[8]) {
   return make_uint4(v[0] | ((uint32_t)v[1] << 16), v[2] | ((uint32_t)v[3] << 16),
                     v[4] | ((uint32_t)v[5] << 16), v[6] | ((uint32_t)v[7] << 16));
 }
+// two fp32 -> packed bf16 pair (RNE; a in the low half), one conversion instruction
+__device__ __forceinline__ uint32_t bf16x2(float a, float b) {
+  const __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<const uint32_t*>(&v);
+}
 // 8 fp32 -> bf16 hi (and lo = bf16(x - hi) if lo != nullptr) at operand chunk (row, ch)
 __device__ __forceinline__ void put8(uint8_t* hi, uint8_t* lo, int row, int ch, const float (&f)[8]) {
-  uint16_t h[8], l[8];
+  uint32_t h[4], l[4];
 #pragma unroll
-  for (int j = 0; j < 8; ++j) {
-    h[j] = f32_to_bf16_rne(f[j]);
-    l[j] = f32_to_bf16_rne(f[j] - bf16_bits_to_f32(h[j]));
+  for (int j = 0; j < 4; ++j) {
+    h[j] = bf16x2(f[2 * j], f[2 * j + 1]);
+    l[j] = bf16x2(f[2 * j] - __uint_as_float(h[j] << 16), f[2 * j + 1] - __uint_as_float(h[j] & 0xffff0000u));
   }
   const uint32_t o = chunk_off(row, ch);
-  *reinterpret_cast<uint4*>(hi + o) = pack8(h);
-  if (lo) *reinterpret_cast<uint4*>(lo + o) = pack8(l);
+  *reinterpret_cast<uint4*>(hi + o) = make_uint4(h[0], h[1], h[2], h[3]);
+  if (lo) *reinterpret_cast<uint4*>(lo + o) = make_uint4(l[0], l[1], l[2], l[3]);
 }
 __device__ __forceinline__ void get8(const uint8_t* op, int row, int ch, float (&f)[8]) {
   unpack8(*reinterpret_cast<const uint4*>(op + chunk_off(row, ch)), f);
@@ -485,7 +490,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         const int fi = i / F, k = i - fi * F;
         float g = 0.f;
         for (int m = 0; m < nm; ++m) g = fmaf(Ds[m * F + fi], Rs[m * F + k], g);
-        G[p.off[7] + i] += g;
+        G[p.off[7] + i] = g;   // zeroed at the tile start: 0 + g
       }
       // dr_m[k] = sum_f W1[f][k] da_m[f] (f order): dh^T of every atom of m
       for (int mb = 8 * half; mb < nm; mb += 16) {
@@ -653,7 +658,7 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
         if (tid < F)
           for (int vv = 0; vv < na; ++vv) Es[(int)p.atom_type[a0 + vv] * F + tid] += Hs[vv * (F + 1) + tid];
         __syncthreads();
-        for (int i = tid; i < n_types * F; i += kThreads) G[p.off[0] + i] += Es[i];
+        for (int i = tid; i < n_types * F; i += kThreads) G[p.off[0] + i] = Es[i];   // zeroed: 0 + sum
       } else {
         // more than 128 atom types: the per-type sums do not fit op2; accumulate
         // in the (zeroed) partial directly, same order
