@@ -603,7 +603,10 @@ __global__ void __launch_bounds__(kThreads, 1) mpnn_train_tile_kernel(MpnnTrainP
           for (int j = 0; j < 64; ++j) Gm[(tc0 + j) * F + k] = g64[j];
         } else {
 #pragma unroll
-          for (int j = 0; j < 64; ++j) Gm[(tc0 + j) * F + k] += g64[j];
+          // fire-and-forget reductions (red.global.add.f32): this thread is the only
+          // writer of these elements, so they apply in program order, the same
+          // sequence of fp32 adds as a load-add-store, without the round trip
+          for (int j = 0; j < 64; ++j) atomicAdd(&Gm[(tc0 + j) * F + k], g64[j]);
         }
       };
       flush(G + p.off[5], t == p.T - 1);                            // dU
