@@ -141,9 +141,16 @@ __device__ void gather(uint8_t* out_hi, uint8_t* out_lo, const uint8_t* src_hi, 
     if (!trans) {
       put8(out_hi, out_lo, v, ch, acc);
     } else {
+      // column v of the transposed operand: lanes l and l + 16 hold rows v and
+      // v + 1 (v even: i = 16 v + ch, 32 consecutive i per warp), one 32-bit
+      // word per (f, v pair)
+      const int lane = tid & 31;
 #pragma unroll
-      for (int j = 0; j < 8; ++j)
-        *reinterpret_cast<uint16_t*>(out_hi + elem_off(8 * ch + j, v)) = f32_to_bf16_rne(acc[j]);
+      for (int j = 0; j < 8; ++j) {
+        const uint32_t b0 = f32_to_bf16_rne(acc[j]);
+        const uint32_t b1 = __shfl_down_sync(0xffffffffu, b0, 16);
+        if (lane < 16) *reinterpret_cast<uint32_t*>(out_hi + elem_off(8 * ch + j, v)) = b0 | (b1 << 16);
+      }
     }
   }
 }
