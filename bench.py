@@ -79,7 +79,8 @@ class ClockSampler:
         os.makedirs(os.path.dirname(self.path), exist_ok=True)
         q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,"
+             "utilization.memory")
         try:
             self.f = open(self.path, "w")
             self.proc = subprocess.Popen(["nvidia-smi", "-i", ",".join(map(str, self.gpus)),
@@ -99,7 +100,7 @@ class ClockSampler:
     def summary(self):
         if not self.proc:
             return None
-        sm, mx_, reasons = [], None, set()
+        sm, mx_, reasons, mem = [], None, set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         try:
             for line in open(self.path):
@@ -111,12 +112,22 @@ class ClockSampler:
                 for n, v in zip(names, c[5:9]):
                     if v.lower().startswith("active"):
                         reasons.add(n)
+                if len(c) >= 10:
+                    try:
+                        mem.append(float(c[9]))
+                    except ValueError:
+                        pass
         except Exception:
             return None
         if not sm:
             return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx_, "reasons": sorted(reasons),
-                "samples": len(sm), "gpus": self.gpus}
+        out = {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx_, "reasons": sorted(reasons),
+               "samples": len(sm), "gpus": self.gpus}
+        if mem:
+            # nvidia-smi utilization.memory: % of time device memory was being read or
+            # written (a coarse hardware-side check of the HBM-bound step; nsys is absent)
+            out["mem_busy_pct_median"] = statistics.median(mem)
+        return out
 
 
 # ---------------------------------------------------------------------------
